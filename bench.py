@@ -1,0 +1,376 @@
+#!/usr/bin/env python
+"""bench.py — snapshot GB/s of the PCcheck path on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl reference]
+
+A step is one whole checkpoint through pccheck.h — every row of SURVEY §8(a): the U-gate
+event, Listing 1 lines 3-11, K1 (gather-pack + CRC32C into the HBM ring), the finalize
+kernel (chunk CRCs + slice digest), copy-engine D2H straight into the registered DRAM
+file mapping (/dev/shm), header COMPLETE, the CAS commit and the pointer record, plus
+(N > 1) the NCCL allreduce(MIN) global commit.  K checkpoints are issued back to back
+with N = 2 in flight and the clock stops when the last one committed.
+
+value = state bytes of the whole job / time (box GB/s; per GPU = value / n_gpus).
+e2e   = the same with the state re-uploaded from pinned host memory every step.
+Rank 0 prints ONE JSON line.  --impl reference times the CPU oracle (oracle/) instead.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "snapshot GB/s per GPU & box at 1/2/4/8 B200; % iter slowdown @ ckpt every 10 iters"
+WORKLOADS = {
+    "c1": "synthetic 64 MiB fp32 state in 97 mixed-size tensors, 4 MiB chunks, 2 in-flight checkpoints, DRAM-file target",
+    "c2": "VGG-16 fp32 params + SGD momentum (1.107 GB), 64 MiB chunks, 2 in-flight checkpoints, DRAM-file target",
+    "c3": "OPT-1.3B fp32 params + Adam (15.79 GB), 64 MiB chunks, 4 in-flight checkpoints, DRAM-file target",
+    "c4": "BLOOM-7b1 bf16 params + fp32 master + Adam (98.97 GB), 64 MiB chunks, 1/world slice per rank",
+}
+
+
+def env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons DURING the timed region (B200_PROFILING.md)."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in self.lines:
+            p = [x.strip() for x in l.split(",")]
+            if len(p) < 8:
+                continue
+            try:
+                sm.append(float(p[1]))
+                mx.append(float(p[2]))
+            except ValueError:
+                continue
+            for n, v in zip(names, p[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def d2h_peak_gbs(torch, nbytes=1 << 30):
+    """Pinned cudaMemcpy D2H peak, measured live (the link roofline denominator)."""
+    d = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    h = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    s = torch.cuda.Stream()
+    best = 1e9
+    with torch.cuda.stream(s):
+        for i in range(5):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(s)
+            h.copy_(d, non_blocking=True)
+            b.record(s)
+            b.synchronize()
+            if i >= 1:
+                best = min(best, a.elapsed_time(b))
+    del d, h
+    return nbytes / (best * 1e-3) / 1e9
+
+
+def cpu_baseline(specs, state, cb, budget_s=12.0):
+    """The oracle as it stands (single-threaded C, byte-at-a-time CRC), on a bounded sample:
+    whole chunks of the same image, as many as fit in ~budget_s of CPU work."""
+    import oracle
+    from synth import host_bytes
+    hb = [host_bytes(t) for t in state]
+    nb = [s.nbytes for s in specs]
+    off, end, c = oracle.layout(nb, 256, cb)
+    done, t0 = 0, time.perf_counter()
+    while done < c and time.perf_counter() - t0 < budget_s:
+        img = oracle.pack(hb, 256, cb, first_chunk=done, count=1)
+        oracle.chunk_crcs(img, cb)
+        done += 1
+    dt = time.perf_counter() - t0
+    return {"value": done * cb / dt / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": f"pack + CRC32C of the first {done} of {c} {cb >> 20} MiB chunks of the same image "
+                      f"({done * cb / 1e9:.3f} GB, {dt:.1f} s, single-threaded plain C)"}
+
+
+def load_traffic(name):
+    p = os.path.join(ROOT, "profiles", "k1_traffic.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(name)
+    except Exception:
+        return None
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle on the same workload, bounded sample per step."""
+    if rank != 0:
+        return
+    import oracle  # noqa: F401  (reference arm: the one other place bench.py runs oracle/)
+    from synth import config_tensors
+    import torch
+    specs = config_tensors(args.config)
+    cb = 64 << 20 if args.config != "c1" else 4 << 20
+    from synth import make_state
+    state = make_state(specs, "cpu", seed=0, it=0)
+    import oracle as O
+    hb = [t.reshape(-1).view(torch.uint8).numpy() if t.dim() else t.reshape(1).view(torch.uint8).numpy()
+          for t in state]
+    nb = [s.nbytes for s in specs]
+    off, end, c = O.layout(nb, 256, cb)
+    per_step = max(1, min(c, 2))
+    times = []
+    j = 0
+    for step in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        img = O.pack(hb, 256, cb, first_chunk=j % c, count=min(per_step, c - j % c))
+        O.chunk_crcs(img, cb)
+        dt = time.perf_counter() - t0
+        if step >= args.warmup:
+            times.append((img.nbytes, dt))
+        j += per_step
+    tot_b = sum(b for b, _ in times)
+    tot_t = sum(t for _, t in times)
+    v = tot_b / tot_t / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "GB/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_t / len(times) * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u8",
+            "data": "synthetic (seeded bit patterns shaped like the model state)",
+            "config": {"workload": WORKLOADS.get(args.config, args.config), "config": args.config,
+                       "chunk_bytes": cb},
+            "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle",
+                             "sample": f"per step: pack + CRC32C of {per_step} {cb >> 20} MiB chunks"},
+            "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c2")
+    ap.add_argument("--impl", default="native", choices=["native", "reference"])
+    ap.add_argument("--inflight", type=int, default=2)
+    ap.add_argument("--no-slowdown", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--mode", default="mapfile", choices=["mapfile", "zerocopy", "nullsink", "pwrite"])
+    args = ap.parse_args()
+    rank, world = env_int("RANK", 0), env_int("WORLD_SIZE", 1)
+    local = env_int("LOCAL_RANK", 0)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    args.warmup = max(3, args.warmup)
+
+    import torch
+    import torch.distributed as dist
+    torch.cuda.set_device(local)
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import paper_conf_asplos_strati0k25_b200 as pcc
+    from synth import config_tensors, make_state
+
+    specs = config_tensors(args.config)
+    cb = 4 << 20 if args.config == "c1" else 64 << 20
+    state = make_state(specs, "cuda", seed=0, it=0)
+    state_bytes = sum(s.nbytes for s in specs)
+    uid = None
+    if world > 1:
+        obj = [pcc.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    flags = {"mapfile": pcc.MAPFILE, "zerocopy": pcc.MAPFILE | pcc.ZEROCOPY, "nullsink": pcc.NULLSINK,
+             "pwrite": pcc.ODIRECT}[args.mode]
+    shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
+    path = None if args.mode == "nullsink" else os.path.join(shm, f"pcc_bench_{os.getpid()}_r{rank}.pcc")
+    ck = pcc.PCCheck(path, chunk_bytes=cb, max_inflight=args.inflight, flags=flags, device=local, rank=rank,
+                     world=world, nccl_unique_id=uid, staging_bytes=8 * cb)
+    ck.register(state)
+    geo = ck.geometry()
+    slice_bytes = geo["count"] * cb
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    it = 0
+
+    def one_ckpt():
+        nonlocal it
+        it += 1
+        h = ck.checkpoint(it, stream)
+        ck.guard(stream)
+        if world > 1:
+            ck.commit()
+        return h
+
+    # ---- warm-up
+    for _ in range(args.warmup):
+        ck.wait(one_ckpt())
+    if world > 1:
+        ck.commit()
+    barrier()
+
+    # ---- timed region: K checkpoints, N in flight
+    clocks = ClockSampler(local)
+    clocks.start()
+    launches0 = ck.kernel_launches()
+    barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t0 = time.perf_counter()
+    e0.record(stream)
+    hs = [one_ckpt() for _ in range(args.steps)]
+    for h in hs:
+        ck.wait(h)
+    if world > 1:
+        ck.commit()
+    e1.record(stream)
+    e1.synchronize()
+    wall = time.perf_counter() - t0
+    dev_ms = e0.elapsed_time(e1)
+    launches = ck.kernel_launches() - launches0
+    clk = clocks.stop()
+    infos = [ck.info(h) for h in hs]
+    pack_ms = statistics.mean(i["pack_ms"] for i in infos)
+    fin_ms = statistics.mean(i["finalize_ms"] for i in infos)
+    lat_ms = statistics.median((i["t_committed_us"] - i["t_call_us"]) / 1e3 for i in infos)
+    t = torch.tensor([dev_ms], device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_total = float(t.item())
+    value = state_bytes * args.steps / (ms_total * 1e-3) / 1e9  # whole job (every rank packs its 1/W slice)
+
+    # ---- e2e: the state comes from pinned host memory every step (H2D inside the timed region)
+    host_state = [torch.empty_like(s, device="cpu").pin_memory() for s in state]
+    for h_, d_ in zip(host_state, state):
+        h_.copy_(d_)
+    barrier()
+    e2 = torch.cuda.Event(enable_timing=True)
+    e3 = torch.cuda.Event(enable_timing=True)
+    e2.record(stream)
+    hs2 = []
+    for _ in range(args.steps):
+        for h_, d_ in zip(host_state, state):
+            d_.copy_(h_, non_blocking=True)
+        hs2.append(one_ckpt())
+    crc_bytes = 0
+    for h in hs2:
+        ck.wait(h)
+        crc_bytes += 4 * (geo["count"] + 1)
+        ck.info(h, with_crc=True)  # the step's result read (CRC table + digest)
+    if world > 1:
+        ck.commit()
+    e3.record(stream)
+    e3.synchronize()
+    t2 = torch.tensor([e2.elapsed_time(e3)], device="cuda")
+    if world > 1:
+        dist.all_reduce(t2, op=dist.ReduceOp.MAX)
+    e2e_value = state_bytes * args.steps / (float(t2.item()) * 1e-3) / 1e9
+
+    peak_link = d2h_peak_gbs(torch)
+    ck.close()
+    if path and os.path.exists(path):
+        os.unlink(path)
+
+    slowdown = None
+    if rank == 0 and world == 1 and not args.no_slowdown and args.config == "c2":
+        try:
+            from tools.slowdown import vgg16_slowdown
+            slowdown = vgg16_slowdown(pcc, iters=60, every=10)
+        except Exception as ex:  # noqa: BLE001
+            slowdown = {"error": repr(ex)[:200]}
+
+    if rank == 0:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            peaks = json.load(f)
+        k1_bytes = 2 * slice_bytes  # read the slice's state bytes + write the packed slice (R3: pads count)
+        k1_achieved = k1_bytes / (pack_ms * 1e-3) / 1e9
+        link_achieved = slice_bytes / (ms_total * 1e-3 / args.steps) / 1e9
+        cpu = None
+        if not args.no_cpu_baseline:
+            cpu = cpu_baseline(specs, state, cb)
+        line = {
+            "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_total / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "u8",
+            "data": "synthetic (seeded bit patterns; shapes of the model's params + optimizer state)",
+            "config": {"workload": WORKLOADS.get(args.config, args.config), "config": args.config,
+                       "state_bytes": state_bytes, "chunk_bytes": cb, "chunks": geo["n_chunks"],
+                       "inflight": args.inflight, "mode": args.mode, "parallelism": f"dp{world}",
+                       "target": "DRAM file on /dev/shm (tmpfs), mmap + cudaHostRegister" if args.mode != "nullsink"
+                       else "null sink", "l2": "inputs larger than L2 (state >> 126 MB)"},
+            "per_gpu_gbs": value / world,
+            "checkpoint_latency_ms_p50": lat_ms,
+            "roofline": {"bound": "hbm", "kernel": "k_snapshot<pack> (K1)", "achieved": k1_achieved,
+                         "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": k1_achieved / peaks["hbm_gbs"],
+                         "traffic": load_traffic(f"{args.config}_k1"),
+                         "algorithmic_bytes_per_launch": k1_bytes, "launch_ms": pack_ms,
+                         "peak_source": "MEASURED_PEAKS.json hbm_gbs (burst copy)"},
+            "link_roofline": {"bound": "pcie_d2h", "achieved": link_achieved, "peak": peak_link, "unit": "GB/s",
+                              "frac": link_achieved / peak_link,
+                              "peak_source": "pinned 1 GiB cudaMemcpy D2H, measured in this run"},
+            "finalize_ms": fin_ms,
+            "cpu_baseline": cpu,
+            "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": state_bytes,
+                    "d2h_bytes_per_step": slice_bytes + 4 * (geo["count"] + 1)},
+            "gpu_launches": launches,
+            "clocks": clk,
+            "slowdown": slowdown,
+            "wall_s_timed": wall,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

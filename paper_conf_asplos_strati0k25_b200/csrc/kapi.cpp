@@ -1,0 +1,146 @@
+// kapi.cpp — pccheck_kernels.h: K1 / K2 on caller buffers (no manager, no file).
+#include <cuda_runtime.h>
+
+#include <cstring>
+
+#include "../../include/pccheck_kernels.h"
+#include "errors.hpp"
+#include "kernels.hpp"
+#include "layout.hpp"
+
+namespace pcc {
+int cuda_error(cudaError_t e, const char *what);  // runtime.cpp
+}
+
+using namespace pcc;
+
+namespace {
+
+struct Scratch {
+    SegRow *rows = nullptr;
+    uint32_t *row_begin = nullptr, *tile_crc = nullptr, *scratch = nullptr, *crc_tmp = nullptr;
+    DevGeometry geom;
+    ~Scratch() {
+        cudaFree(rows);
+        cudaFree(row_begin);
+        cudaFree(tile_crc);
+        cudaFree(scratch);
+        cudaFree(crc_tmp);
+        free_geometry(&geom);
+    }
+};
+
+int prepare(const pcc_tensor *t, uint32_t n, uint32_t align, uint64_t cb, uint64_t first, uint64_t count,
+            cudaStream_t s, HostLayout *L, Scratch *S, SnapParams *P) {
+    if ((n && !t) || count == 0) return count == 0 ? PCC_OK : set_error(PCC_EINVAL, "null tensor table");
+    int rc = build_layout(t, n, align ? align : 256, cb, first, (int64_t)count, L);
+    if (rc) return set_error(PCC_EINVAL, "bad geometry");
+    if (first + count > L->C) return set_error(PCC_EINVAL, "chunk range beyond the image");
+    cudaError_t e;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const CrcTables *tb;
+    const CrcConsts *cs;
+    if ((e = device_tables(dev, &tb, &cs)) != cudaSuccess) return cuda_error(e, "tables");
+    if ((e = setup_geometry(&S->geom, cb, (uint32_t)count, s)) != cudaSuccess) return cuda_error(e, "geometry");
+    const size_t nrows = L->rows.size() ? L->rows.size() : 1;
+    if ((e = cudaMalloc(&S->rows, nrows * sizeof(SegRow))) != cudaSuccess) return cuda_error(e, "rows");
+    if ((e = cudaMalloc(&S->row_begin, (count + 1) * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "rb");
+    if ((e = cudaMalloc(&S->tile_crc, count * S->geom.tpc * sizeof(uint32_t))) != cudaSuccess)
+        return cuda_error(e, "tile crc");
+    if ((e = cudaMalloc(&S->scratch, 4 * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "scratch");
+    if (!L->rows.empty())
+        cudaMemcpyAsync(S->rows, L->rows.data(), L->rows.size() * sizeof(SegRow), cudaMemcpyHostToDevice, s);
+    cudaMemcpyAsync(S->row_begin, L->row_begin.data(), (count + 1) * sizeof(uint32_t), cudaMemcpyHostToDevice, s);
+    cudaMemsetAsync(S->scratch, 0, 4 * sizeof(uint32_t), s);
+    // host staging vectors must outlive the async copies
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_error(e, "upload");
+    P->rows = S->rows;
+    P->row_begin = S->row_begin;
+    P->chunk_bytes = cb;
+    P->first = 0;
+    P->count = (uint32_t)count;
+    P->tpc = S->geom.tpc;
+    P->ring_head = 0;
+    P->ring_slots = count;
+    P->tile_crc = S->tile_crc;
+    P->tables = tb;
+    P->consts = cs;
+    return PCC_OK;
+}
+
+}  // namespace
+
+extern "C" int pcc_k_layout(const pcc_tensor *t, uint32_t n, uint32_t align, uint64_t chunk_bytes, uint64_t *off,
+                            uint64_t *end_bytes, uint64_t *n_chunks) {
+    HostLayout L;
+    int rc = build_layout(t, n, align ? align : 256, chunk_bytes, 0, 0, &L);
+    if (rc) return rc;
+    if (off) std::memcpy(off, L.off.data(), n * sizeof(uint64_t));
+    if (end_bytes) *end_bytes = L.end;
+    if (n_chunks) *n_chunks = L.C;
+    return PCC_OK;
+}
+
+extern "C" int pcc_k_pack(const pcc_tensor *t, uint32_t n, uint32_t align, uint64_t chunk_bytes,
+                          uint64_t first_chunk, uint64_t count, void *dst, uint32_t *crc, uint32_t *digest,
+                          void *stream) {
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    HostLayout L;
+    Scratch S;
+    SnapParams P{};
+    int rc = prepare(t, n, align, chunk_bytes, first_chunk, count, s, &L, &S, &P);
+    if (rc || count == 0) return rc;
+    P.ring_base = static_cast<char *>(dst);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaError_t e = launch_pack(P, snapshot_grid(dev, (uint32_t)(count * P.tpc), 0), s);
+    if (e != cudaSuccess) return cuda_error(e, "K1 launch");
+    FinalizeParams F{};
+    F.tile_crc = S.tile_crc;
+    F.n = (uint32_t)count;
+    F.tpc = P.tpc;
+    F.tile_shift = S.geom.tile_shift;
+    F.chunk_shift = S.geom.chunk_shift;
+    F.ff = S.geom.ff;
+    F.crc_out = crc;
+    F.scratch = S.scratch;
+    if ((e = launch_finalize(F, s)) != cudaSuccess) return cuda_error(e, "finalize launch");
+    cudaMemcpyAsync(digest, S.scratch + 3, 4, cudaMemcpyDeviceToDevice, s);
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_error(e, "K1");
+    return PCC_OK;
+}
+
+extern "C" int pcc_k_unpack(const pcc_tensor *t, uint32_t n, uint32_t align, uint64_t chunk_bytes,
+                            uint64_t first_chunk, uint64_t count, const void *src, const uint32_t *expect,
+                            uint32_t *bad, uint32_t *n_bad, uint32_t *digest, void *stream) {
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    HostLayout L;
+    Scratch S;
+    SnapParams P{};
+    int rc = prepare(t, n, align, chunk_bytes, first_chunk, count, s, &L, &S, &P);
+    if (rc || count == 0) return rc;
+    P.ring_base = const_cast<char *>(static_cast<const char *>(src));
+    cudaError_t e;
+    if ((e = cudaMalloc(&S.crc_tmp, count * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "crc tmp");
+    int dev = 0;
+    cudaGetDevice(&dev);
+    e = launch_unpack(P, snapshot_grid(dev, (uint32_t)(count * P.tpc), 0), s);
+    if (e != cudaSuccess) return cuda_error(e, "K2 launch");
+    FinalizeParams F{};
+    F.tile_crc = S.tile_crc;
+    F.n = (uint32_t)count;
+    F.tpc = P.tpc;
+    F.tile_shift = S.geom.tile_shift;
+    F.chunk_shift = S.geom.chunk_shift;
+    F.ff = S.geom.ff;
+    F.crc_out = S.crc_tmp;
+    F.expect = expect;
+    F.bad = bad;
+    F.scratch = S.scratch;
+    if ((e = launch_finalize(F, s)) != cudaSuccess) return cuda_error(e, "finalize launch");
+    cudaMemcpyAsync(n_bad, S.scratch + 2, 4, cudaMemcpyDeviceToDevice, s);
+    cudaMemcpyAsync(digest, S.scratch + 3, 4, cudaMemcpyDeviceToDevice, s);
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_error(e, "K2");
+    return PCC_OK;
+}

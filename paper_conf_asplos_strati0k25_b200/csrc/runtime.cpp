@@ -1,0 +1,1161 @@
+// runtime.cpp — the PCcheck manager on one B200 (pccheck.h).
+//
+// PAPER.md Fig 5 (L117) / §3.1 L125-L141 on B200, one process per GPU:
+//   training thread   pcc_checkpoint: Listing 1 lines 3-11 (CommitEngine::begin), then K1
+//                     on the pack stream: the registered tensors -> the HBM chunk ring with
+//                     CRC32C (the "extra copy of the weights" of L139, affordable in 180 GB,
+//                     so the U-gate only waits for an HBM->HBM pack, not for PCIe)
+//   orchestrator      one thread: FILLING header, then per chunk a copy-engine D2H from the
+//                     ring into host DRAM (L164: copy engines, pinned memory) — straight into
+//                     the registered file mapping (PCC_MAPFILE) or a pinned staging slot
+//   persist pool      p threads (L168, L176): wait for the chunk's copy, pwrite it to the
+//                     slot (PWRITE mode), recycle ring / staging; the last chunk runs
+//                     Listing 1 lines 16-34 (CommitEngine::complete)
+// Chunks of a checkpoint land contiguously in their slot (L127, L281: "contiguous on
+// storage"), N checkpoints may be in flight (L139, Fig 6), copy and persist overlap per
+// chunk (L141, Fig 7).
+#include <cuda_runtime.h>
+#include <fcntl.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cerrno>
+#include <chrono>
+#include <condition_variable>
+#include <cstdlib>
+#include <cstring>
+#include <deque>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../include/pccheck.h"
+#include "commit.hpp"
+#include "errors.hpp"
+#include "kernels.hpp"
+#include "layout.hpp"
+#include "nccl_shim.hpp"
+
+namespace pcc {
+
+int cuda_error(cudaError_t e, const char *what) {
+    char b[512];
+    std::snprintf(b, sizeof b, "%s: %s", what, cudaGetErrorString(e));
+    err_state().msg = b;
+    return -PCC_ECUDA;
+}
+
+using Clock = std::chrono::steady_clock;
+
+struct Launch {
+    uint32_t first, count;
+    cudaEvent_t ev;
+};
+
+struct Ckpt {
+    Ticket t;
+    std::atomic<int> state{PCC_ST_QUEUED};
+    std::atomic<int> err{0};
+    uint64_t ring_start = 0;
+    std::mutex mu;
+    std::condition_variable cv;
+    std::vector<Launch> launches;
+    uint32_t launched = 0;  // chunks launched (guarded by mu)
+    bool launch_failed = false;
+    std::atomic<uint32_t> remaining{0};
+    cudaEvent_t ev_train = nullptr, ev_begin = nullptr, ev_packed = nullptr, ev_final = nullptr;
+    double t_call = 0, t_packed = 0, t_landed = 0, t_persisted = 0, t_committed = 0;
+    float pack_ms = 0, fin_ms = 0;
+    uint32_t digest = 0;
+    std::vector<uint32_t> crc;
+};
+
+struct PersistTask {
+    std::shared_ptr<Ckpt> ck;
+    uint32_t j;
+    char *dest;  // host address of the chunk (staging slot or file mapping)
+    cudaEvent_t ev;
+    bool pooled_ev;
+};
+
+template <class T>
+class BlockingQueue {
+   public:
+    void push(T v) {
+        {
+            std::lock_guard<std::mutex> lk(mu_);
+            q_.push_back(std::move(v));
+        }
+        cv_.notify_one();
+    }
+    bool pop(T *out) {  // false on close
+        std::unique_lock<std::mutex> lk(mu_);
+        cv_.wait(lk, [&] { return closed_ || !q_.empty(); });
+        if (q_.empty()) return false;
+        *out = std::move(q_.front());
+        q_.pop_front();
+        return true;
+    }
+    void close() {
+        {
+            std::lock_guard<std::mutex> lk(mu_);
+            closed_ = true;
+        }
+        cv_.notify_all();
+    }
+
+   private:
+    std::mutex mu_;
+    std::condition_variable cv_;
+    std::deque<T> q_;
+    bool closed_ = false;
+};
+
+}  // namespace pcc
+
+using namespace pcc;
+
+struct pcc_ctx {
+    pcc_config cfg{};
+    std::string path;
+    int device = 0;
+    Clock::time_point t0;
+    cudaStream_t pack_stream = nullptr, copy_stream = nullptr, aux_stream = nullptr;
+    cudaEvent_t ev_guard = nullptr;
+    bool guard_armed = false;
+    const CrcTables *tables = nullptr;
+    const CrcConsts *consts = nullptr;
+    std::atomic<uint64_t> launches{0};
+
+    // registration
+    bool registered = false;
+    std::vector<pcc_tensor> tensors;
+    std::vector<std::string> names;
+    HostLayout layout;
+    uint64_t first = 0, n = 0;
+    SegRow *rows_dev = nullptr;
+    uint32_t *row_begin_dev = nullptr;
+    DevGeometry geom;
+    SlotGeom sgeom{};
+    uint32_t lcrc = 0;
+    uint32_t n_slots = 0;
+    // per storage slot scratch (a slot belongs to at most one checkpoint in flight)
+    std::vector<uint32_t *> tile_crc_dev, crc_dev, scratch_dev;
+    std::vector<uint32_t *> crc_host;  // pinned [n + 1] (+ digest)
+
+    // HBM ring (Variant B)
+    char *ring = nullptr;
+    uint64_t ring_slots = 0, ring_head = 0, ring_tail = 0;
+    std::vector<uint8_t> ring_done;
+    std::mutex ring_mu;
+    std::condition_variable ring_cv;
+
+    // pinned staging pool (PWRITE / NULLSINK)
+    char *staging = nullptr;
+    uint64_t staging_slots = 0;
+    std::vector<char *> staging_free;
+    std::mutex st_mu;
+    std::condition_variable st_cv;
+
+    // file
+    int fd = -1;
+    bool odirect = false;
+    char *map = nullptr;
+    uint64_t map_bytes = 0;
+    char *map_dev = nullptr;
+
+    std::unique_ptr<CommitEngine> engine;
+    std::mutex ck_mu;
+    std::condition_variable ck_cv;
+    std::map<uint64_t, std::shared_ptr<Ckpt>> ckpts;  // handle (= counter) -> record
+
+    // threads
+    BlockingQueue<std::shared_ptr<Ckpt>> jobs;
+    BlockingQueue<PersistTask> tasks;
+    std::thread orchestrator;
+    std::vector<std::thread> persisters;
+    std::mutex evpool_mu;
+    std::vector<cudaEvent_t> evpool;
+
+    // NCCL (world > 1)
+    NcclComm nccl;
+    int64_t *red_dev = nullptr;
+    int64_t *red_host = nullptr;
+
+    double now_us() const { return std::chrono::duration<double, std::micro>(Clock::now() - t0).count(); }
+    bool mapfile() const { return cfg.flags & PCC_MAPFILE; }
+    bool nullsink() const { return cfg.flags & PCC_NULLSINK; }
+    bool zerocopy() const { return cfg.flags & PCC_ZEROCOPY; }
+    uint64_t cb() const { return cfg.chunk_bytes; }
+    uint64_t slot_data_off(uint32_t s) const { return slot_offset(s, n, cb()) + header_bytes(n); }
+};
+
+namespace {
+
+cudaEvent_t get_event(pcc_ctx *c) {
+    {
+        std::lock_guard<std::mutex> lk(c->evpool_mu);
+        if (!c->evpool.empty()) {
+            cudaEvent_t e = c->evpool.back();
+            c->evpool.pop_back();
+            return e;
+        }
+    }
+    cudaEvent_t e = nullptr;
+    cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    return e;
+}
+
+void put_event(pcc_ctx *c, cudaEvent_t e) {
+    std::lock_guard<std::mutex> lk(c->evpool_mu);
+    c->evpool.push_back(e);
+}
+
+void set_state(pcc_ctx *c, Ckpt *ck, int st) {
+    {
+        std::lock_guard<std::mutex> lk(c->ck_mu);
+        ck->state.store(st);
+    }
+    c->ck_cv.notify_all();
+}
+
+void ring_release(pcc_ctx *c, uint64_t idx) {
+    {
+        std::lock_guard<std::mutex> lk(c->ring_mu);
+        c->ring_done[idx % c->ring_slots] = 1;
+        while (c->ring_tail < c->ring_head && c->ring_done[c->ring_tail % c->ring_slots]) {
+            c->ring_done[c->ring_tail % c->ring_slots] = 0;
+            ++c->ring_tail;
+        }
+    }
+    c->ring_cv.notify_all();
+}
+
+char *staging_acquire(pcc_ctx *c) {
+    std::unique_lock<std::mutex> lk(c->st_mu);
+    c->st_cv.wait(lk, [&] { return !c->staging_free.empty(); });
+    char *p = c->staging_free.back();
+    c->staging_free.pop_back();
+    return p;
+}
+
+void staging_release(pcc_ctx *c, char *p) {
+    {
+        std::lock_guard<std::mutex> lk(c->st_mu);
+        c->staging_free.push_back(p);
+    }
+    c->st_cv.notify_one();
+}
+
+int pwrite_full(int fd, const char *p, uint64_t n, uint64_t off) {
+    while (n) {
+        ssize_t w = ::pwrite(fd, p, n, (off_t)off);
+        if (w < 0) {
+            if (errno == EINTR) continue;
+            return set_errno_error("pwrite chunk", errno);
+        }
+        p += w;
+        n -= (uint64_t)w;
+        off += (uint64_t)w;
+    }
+    return PCC_OK;
+}
+
+void fail_ckpt(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck, int err) {
+    int expected = 0;
+    ck->err.compare_exchange_strong(expected, err);
+}
+
+// Listing 1 lines 16-34 for a checkpoint whose chunks are all durable.
+void finish_ckpt(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
+    cudaError_t e = cudaEventSynchronize(ck->ev_final);
+    if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "finalize"));
+    cudaEventElapsedTime(&ck->pack_ms, ck->ev_begin, ck->ev_packed);
+    cudaEventElapsedTime(&ck->fin_ms, ck->ev_packed, ck->ev_final);
+    const uint32_t *h = c->crc_host[ck->t.slot];
+    ck->crc.assign(h, h + c->n);
+    ck->digest = h[c->n];
+    ck->t_persisted = c->now_us();
+    if (ck->err.load()) {
+        c->engine->fail(ck->t);
+        set_state(c, ck.get(), PCC_ST_FAILED);
+        return;
+    }
+    if (c->fd >= 0 && (c->cfg.flags & PCC_FSYNC) && ::fdatasync(c->fd) != 0) {
+        fail_ckpt(c, ck, set_errno_error("fdatasync", errno));
+        c->engine->fail(ck->t);
+        set_state(c, ck.get(), PCC_ST_FAILED);
+        return;
+    }
+    set_state(c, ck.get(), PCC_ST_PERSISTED);
+    int st = PCC_ST_FAILED;
+    int rc = c->engine->complete(ck->t, ck->crc.data(), ck->digest, &st);
+    if (rc) fail_ckpt(c, ck, rc);
+    if (c->cfg.world == 1 || st == PCC_ST_FAILED) {
+        ck->t_committed = c->now_us();
+        set_state(c, ck.get(), st);
+    }
+    // world > 1: the engine's on_state callback moves it to LOCAL_COMMIT in counter order
+}
+
+void persist_loop(pcc_ctx *c) {
+    cudaSetDevice(c->device);
+    PersistTask task;
+    while (c->tasks.pop(&task)) {
+        Ckpt *ck = task.ck.get();
+        cudaError_t e = cudaEventSynchronize(task.ev);
+        if (e != cudaSuccess) fail_ckpt(c, task.ck, cuda_error(e, "chunk copy"));
+        if (task.pooled_ev) put_event(c, task.ev);
+        if (!c->zerocopy()) ring_release(c, ck->ring_start + task.j);
+        const double t = c->now_us();
+        if (!c->mapfile()) {
+            if (!c->nullsink() && !ck->err.load()) {
+                int rc = pwrite_full(c->fd, task.dest, c->cb(), c->slot_data_off(ck->t.slot) + task.j * c->cb());
+                if (rc) fail_ckpt(c, task.ck, rc);
+            }
+            staging_release(c, task.dest);
+        }
+        {
+            std::lock_guard<std::mutex> lk(ck->mu);
+            ck->t_landed = std::max(ck->t_landed, t);
+        }
+        if (ck->remaining.fetch_sub(1) == 1) finish_ckpt(c, task.ck);
+    }
+}
+
+void orchestrate_loop(pcc_ctx *c) {
+    cudaSetDevice(c->device);
+    std::shared_ptr<Ckpt> ck;
+    while (c->jobs.pop(&ck)) {
+        if (c->fd >= 0) {
+            int rc = c->engine->filling(ck->t);  // R18: before any data byte of this slot changes
+            if (rc) fail_ckpt(c, ck, rc);
+        }
+        size_t li = 0;
+        for (uint32_t j = 0; j < c->n; ++j) {
+            Launch L;
+            {
+                std::unique_lock<std::mutex> lk(ck->mu);
+                ck->cv.wait(lk, [&] { return ck->launched > j || ck->launch_failed; });
+                if (ck->launch_failed && ck->launched <= j) break;
+                while (!(j >= ck->launches[li].first && j < ck->launches[li].first + ck->launches[li].count)) ++li;
+                L = ck->launches[li];
+            }
+            PersistTask task{ck, j, nullptr, nullptr, false};
+            if (c->zerocopy()) {
+                task.ev = L.ev;  // K1 stored the chunk straight into the file mapping
+                task.dest = c->map + c->slot_data_off(ck->t.slot) + (uint64_t)j * c->cb();
+            } else {
+                if (j == L.first) cudaStreamWaitEvent(c->copy_stream, L.ev, 0);
+                task.dest = c->mapfile() ? c->map + c->slot_data_off(ck->t.slot) + (uint64_t)j * c->cb()
+                                         : staging_acquire(c);
+                const char *src = c->ring + ((ck->ring_start + j) % c->ring_slots) * c->cb();
+                cudaError_t e = cudaMemcpyAsync(task.dest, src, c->cb(), cudaMemcpyDeviceToHost, c->copy_stream);
+                if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "D2H"));
+                task.ev = get_event(c);
+                task.pooled_ev = true;
+                cudaEventRecord(task.ev, c->copy_stream);
+            }
+            c->tasks.push(task);
+        }
+        if (c->n == 0) finish_ckpt(c, ck);
+    }
+}
+
+int free_registration(pcc_ctx *c) {
+    cudaFree(c->rows_dev);
+    cudaFree(c->row_begin_dev);
+    c->rows_dev = nullptr;
+    c->row_begin_dev = nullptr;
+    free_geometry(&c->geom);
+    for (auto p : c->tile_crc_dev) cudaFree(p);
+    for (auto p : c->crc_dev) cudaFree(p);
+    for (auto p : c->scratch_dev) cudaFree(p);
+    for (auto p : c->crc_host) cudaFreeHost(p);
+    c->tile_crc_dev.clear();
+    c->crc_dev.clear();
+    c->scratch_dev.clear();
+    c->crc_host.clear();
+    if (c->ring) cudaFree(c->ring);
+    c->ring = nullptr;
+    if (c->staging) cudaFreeHost(c->staging);
+    c->staging = nullptr;
+    c->staging_free.clear();
+    if (c->map) {
+        cudaHostUnregister(c->map);
+        munmap(c->map, c->map_bytes);
+        c->map = nullptr;
+        c->map_dev = nullptr;
+    }
+    c->engine.reset();
+    c->registered = false;
+    return PCC_OK;
+}
+
+void destroy_ckpt_events(pcc_ctx *c, Ckpt *ck) {
+    cudaEventDestroy(ck->ev_train);
+    cudaEventDestroy(ck->ev_begin);
+    cudaEventDestroy(ck->ev_packed);
+    cudaEventDestroy(ck->ev_final);
+    for (auto &L : ck->launches) put_event(c, L.ev);
+    ck->launches.clear();
+}
+
+// keeps the newest kKeep terminal records queryable (pcc_info), frees older ones
+void gc_ckpts(pcc_ctx *c) {
+    constexpr size_t kKeep = 64;
+    std::vector<std::shared_ptr<Ckpt>> dead;
+    {
+        std::lock_guard<std::mutex> lk(c->ck_mu);
+        if (c->ckpts.size() <= kKeep) return;
+        size_t excess = c->ckpts.size() - kKeep;
+        for (auto it = c->ckpts.begin(); it != c->ckpts.end() && excess;) {
+            int s = it->second->state.load();
+            bool term = s == PCC_ST_LOCAL_COMMIT || s == PCC_ST_GLOBAL_COMMIT || s == PCC_ST_OBSOLETE ||
+                        s == PCC_ST_FAILED;
+            if (term && it->second->remaining.load() == 0) {
+                dead.push_back(it->second);
+                it = c->ckpts.erase(it);
+                --excess;
+            } else {
+                ++it;
+            }
+        }
+    }
+    for (auto &ck : dead) destroy_ckpt_events(c, ck.get());
+}
+
+bool any_inflight(pcc_ctx *c) {
+    std::lock_guard<std::mutex> lk(c->ck_mu);
+    for (auto &kv : c->ckpts) {
+        int s = kv.second->state.load();
+        if (s != PCC_ST_LOCAL_COMMIT && s != PCC_ST_GLOBAL_COMMIT && s != PCC_ST_OBSOLETE && s != PCC_ST_FAILED)
+            return true;
+    }
+    return false;
+}
+
+}  // namespace
+
+// ============================================================================ C ABI
+extern "C" {
+
+const char *pcc_strerror(int err) {
+    switch (err < 0 ? -err : err) {
+        case PCC_OK: return "ok";
+        case PCC_EINVAL: return "invalid argument";
+        case PCC_ENOMEM: return "out of memory";
+        case PCC_EBUSY: return "checkpoints in flight";
+        case PCC_EAGAIN: return "try again";
+        case PCC_EIO: return "I/O error";
+        case PCC_ECUDA: return "CUDA error";
+        case PCC_ENCCL: return "NCCL error";
+        case PCC_EORDER: return "iter not strictly increasing";
+        case PCC_ECORRUPT: return "checksum mismatch";
+        case PCC_ELAYOUT: return "layout mismatch";
+        case PCC_ENOENT: return "no valid checkpoint";
+        case PCC_ETIMEDOUT: return "timed out";
+        case PCC_ESTATE: return "invalid state";
+        default: return "unknown error";
+    }
+}
+const char *pcc_last_error(void) { return err_state().msg.c_str(); }
+int pcc_last_errno(void) { return err_state().err_no; }
+
+int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
+    if (!out) return set_error(PCC_EINVAL, "out");
+    *out = nullptr;
+    if (!cfg || cfg->abi_version != PCC_ABI_VERSION) return set_error(PCC_EINVAL, "abi version");
+    if (cfg->chunk_bytes == 0 || cfg->chunk_bytes % 16 || cfg->chunk_bytes >= (1ull << 32) || cfg->max_inflight == 0)
+        return set_error(PCC_EINVAL, "chunk_bytes / max_inflight");
+    if (cfg->world < 1 || cfg->rank < 0 || cfg->rank >= cfg->world) return set_error(PCC_EINVAL, "rank/world");
+    const bool nullsink = cfg->flags & PCC_NULLSINK;
+    if (!nullsink && !cfg->path) return set_error(PCC_EINVAL, "path");
+    if ((cfg->flags & (PCC_MAPFILE | PCC_ODIRECT)) && cfg->chunk_bytes % kPage)
+        return set_error(PCC_EINVAL, "chunk_bytes must be a multiple of 4096 with ODIRECT/MAPFILE");
+    if ((cfg->flags & PCC_ZEROCOPY) && !(cfg->flags & PCC_MAPFILE))
+        return set_error(PCC_EINVAL, "ZEROCOPY needs MAPFILE");
+    if (nullsink && (cfg->flags & PCC_MAPFILE)) return set_error(PCC_EINVAL, "NULLSINK excludes MAPFILE");
+    std::unique_ptr<pcc_ctx> c(new pcc_ctx());
+    c->cfg = *cfg;
+    if (cfg->path) c->path = cfg->path;
+    c->cfg.path = c->path.c_str();
+    if (!c->cfg.align) c->cfg.align = 256;
+    if (c->cfg.align % 16) return set_error(PCC_EINVAL, "align % 16");
+    if (!c->cfg.writer_threads) c->cfg.writer_threads = 4;
+    c->device = cfg->device;
+    c->t0 = Clock::now();
+    cudaError_t e = cudaSetDevice(c->device);
+    if (e != cudaSuccess) return cuda_error(e, "cudaSetDevice");
+    if ((e = device_tables(c->device, &c->tables, &c->consts)) != cudaSuccess) return cuda_error(e, "CRC tables");
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    if ((e = cudaStreamCreateWithPriority(&c->pack_stream, cudaStreamNonBlocking, hi)) != cudaSuccess)
+        return cuda_error(e, "stream");
+    cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking);
+    cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking);
+    cudaEventCreateWithFlags(&c->ev_guard, cudaEventDisableTiming);
+    if (!nullsink) {
+        int flags = O_RDWR | O_CREAT;
+        if ((cfg->flags & PCC_ODIRECT) && !(cfg->flags & PCC_MAPFILE)) flags |= O_DIRECT;
+        c->fd = ::open(c->path.c_str(), flags, 0644);
+        if (c->fd < 0 && (flags & O_DIRECT) && errno == EINVAL) {
+            flags &= ~O_DIRECT;  // filesystem without O_DIRECT: buffered
+            c->fd = ::open(c->path.c_str(), flags, 0644);
+        }
+        if (c->fd < 0) return set_errno_error("open checkpoint file", errno);
+        c->odirect = flags & O_DIRECT;
+    }
+    if (cfg->world > 1) {
+        if (!cfg->nccl_unique_id) return set_error(PCC_EINVAL, "nccl_unique_id required for world > 1");
+        int rc = c->nccl.init(cfg->nccl_unique_id, cfg->world, cfg->rank);
+        if (rc) return rc;
+        cudaMalloc(&c->red_dev, 4 * sizeof(int64_t));
+        cudaMallocHost(&c->red_host, 4 * sizeof(int64_t));
+    }
+    pcc_ctx *raw = c.get();
+    raw->orchestrator = std::thread(orchestrate_loop, raw);
+    for (uint32_t i = 0; i < raw->cfg.writer_threads; ++i) raw->persisters.emplace_back(persist_loop, raw);
+    *out = c.release();
+    return PCC_OK;
+}
+
+int pcc_register(pcc_ctx *c, const pcc_tensor *t, uint32_t nt) {
+    if (!c || (nt && !t)) return set_error(PCC_EINVAL, "args");
+    if (any_inflight(c)) return set_error(PCC_EBUSY, "checkpoints in flight");
+    cudaSetDevice(c->device);
+    free_registration(c);
+    c->tensors.assign(t, t + nt);
+    c->names.clear();
+    for (uint32_t i = 0; i < nt; ++i) {
+        c->names.emplace_back(t[i].name ? t[i].name : "");
+        c->tensors[i].name = nullptr;
+    }
+    HostLayout full;
+    int rc = build_layout(t, nt, c->cfg.align, c->cb(), 0, 0, &full);
+    if (rc) return set_error(PCC_EINVAL, "layout");
+    slice_of(full.C, c->cfg.rank, c->cfg.world, &c->first, &c->n);
+    rc = build_layout(t, nt, c->cfg.align, c->cb(), c->first, (int64_t)c->n, &c->layout);
+    if (rc) return set_error(PCC_EINVAL, "layout slice");
+    std::vector<uint64_t> nb(nt);
+    std::vector<uint32_t> dt(nt);
+    for (uint32_t i = 0; i < nt; ++i) {
+        nb[i] = t[i].nbytes;
+        dt[i] = t[i].dtype;
+    }
+    c->lcrc = layout_crc(nt, nb.data(), dt.data(), c->cfg.align, c->cb());
+    c->sgeom = SlotGeom{c->cb(), (uint32_t)c->cfg.rank, (uint32_t)c->cfg.world, (uint32_t)c->layout.C,
+                        (uint32_t)c->first, (uint32_t)c->n, nt, c->cfg.align, c->lcrc};
+    c->n_slots = c->cfg.max_inflight + 1;
+    cudaError_t e;
+    const size_t nrows = c->layout.rows.empty() ? 1 : c->layout.rows.size();
+    if ((e = cudaMalloc(&c->rows_dev, nrows * sizeof(SegRow))) != cudaSuccess) return cuda_error(e, "rows");
+    if ((e = cudaMalloc(&c->row_begin_dev, (c->n + 1) * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "rb");
+    if (!c->layout.rows.empty())
+        cudaMemcpy(c->rows_dev, c->layout.rows.data(), c->layout.rows.size() * sizeof(SegRow), cudaMemcpyHostToDevice);
+    cudaMemcpy(c->row_begin_dev, c->layout.row_begin.data(), (c->n + 1) * sizeof(uint32_t), cudaMemcpyHostToDevice);
+    if ((e = setup_geometry(&c->geom, c->cb(), (uint32_t)c->n, c->pack_stream)) != cudaSuccess)
+        return cuda_error(e, "geometry");
+    const uint64_t nn = c->n ? c->n : 1;
+    for (uint32_t s = 0; s < c->n_slots; ++s) {
+        uint32_t *a = nullptr, *b = nullptr, *d = nullptr, *h = nullptr;
+        if ((e = cudaMalloc(&a, nn * c->geom.tpc * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "tile crc");
+        if ((e = cudaMalloc(&b, (nn + 1) * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "crc");
+        if ((e = cudaMalloc(&d, 4 * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "scratch");
+        if ((e = cudaMallocHost(&h, (nn + 1) * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "crc host");
+        c->tile_crc_dev.push_back(a);
+        c->crc_dev.push_back(b);
+        c->scratch_dev.push_back(d);
+        c->crc_host.push_back(h);
+    }
+    // HBM ring: default one whole slice (L139's extra copy)
+    if (!c->zerocopy()) {
+        uint64_t r = c->cfg.ring_bytes ? c->cfg.ring_bytes / c->cb() : c->n;
+        if (r == 0) r = 1;
+        if (r > nn) r = nn;
+        c->ring_slots = r;
+        if ((e = cudaMalloc(&c->ring, r * c->cb())) != cudaSuccess) return cuda_error(e, "HBM ring");
+        c->ring_done.assign(r, 0);
+        c->ring_head = c->ring_tail = 0;
+    }
+    // staging pool (c = M / b, L176)
+    if (!c->mapfile()) {
+        uint64_t k = c->cfg.staging_bytes / c->cb();
+        if (k == 0) k = std::max<uint64_t>(2 * c->cfg.writer_threads, 4);
+        if (k > nn) k = nn;
+        c->staging_slots = k;
+        if ((e = cudaHostAlloc(&c->staging, k * c->cb(), cudaHostAllocPortable)) != cudaSuccess)
+            return cuda_error(e, "pinned staging");
+        for (uint64_t i = 0; i < k; ++i) c->staging_free.push_back(c->staging + i * c->cb());
+    }
+    // file: N+1 slots
+    if (c->fd >= 0) {
+        const uint64_t fbytes = file_bytes(c->n_slots, c->n, c->cb());
+        struct stat st;
+        if (fstat(c->fd, &st) == 0 && (uint64_t)st.st_size < fbytes && ftruncate(c->fd, (off_t)fbytes) != 0)
+            return set_errno_error("ftruncate", errno);
+        if (c->mapfile()) {
+            c->map_bytes = fbytes;
+            void *m = mmap(nullptr, fbytes, PROT_READ | PROT_WRITE, MAP_SHARED, c->fd, 0);
+            if (m == MAP_FAILED) return set_errno_error("mmap", errno);
+            c->map = static_cast<char *>(m);
+            if ((e = cudaHostRegister(c->map, fbytes, cudaHostRegisterMapped | cudaHostRegisterPortable)) !=
+                cudaSuccess) {
+                munmap(c->map, fbytes);
+                c->map = nullptr;
+                return cuda_error(e, "cudaHostRegister(file mapping)");
+            }
+            void *dp = nullptr;
+            cudaHostGetDevicePointer(&dp, c->map, 0);
+            c->map_dev = static_cast<char *>(dp);
+        }
+    }
+    c->engine.reset(new CommitEngine());
+    CommitEngine::Config ec;
+    ec.fd = c->fd;
+    ec.geom = c->sgeom;
+    ec.n_inflight = c->cfg.max_inflight;
+    ec.fsync = c->cfg.flags & PCC_FSYNC;
+    ec.on_state = [c](uint64_t counter, int st) {
+        // called under the engine lock; only touches the checkpoint table
+        std::shared_ptr<Ckpt> ck;
+        {
+            std::lock_guard<std::mutex> lk(c->ck_mu);
+            auto it = c->ckpts.find(counter);
+            if (it == c->ckpts.end()) return;
+            ck = it->second;
+            ck->t_committed = c->now_us();
+            ck->state.store(st);
+        }
+        c->ck_cv.notify_all();
+    };
+    if ((rc = c->engine->open(ec))) return rc;
+    if ((e = cudaStreamSynchronize(c->pack_stream)) != cudaSuccess) return cuda_error(e, "register");
+    c->registered = true;
+    return PCC_OK;
+}
+
+static int dp_backpressure(pcc_ctx *c);
+
+int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *out) {
+    if (!c || !out) return set_error(PCC_EINVAL, "args");
+    if (!c->registered) return set_error(PCC_ESTATE, "not registered");
+    cudaStream_t ts = static_cast<cudaStream_t>(train_stream);
+    gc_ckpts(c);
+    auto ck = std::make_shared<Ckpt>();
+    ck->t_call = c->now_us();
+    // Listing 1 lines 3-11
+    if (c->cfg.world > 1) {
+        int rc = dp_backpressure(c);
+        if (rc) return rc;
+    }
+    for (;;) {
+        int rc = c->engine->begin(iter, &ck->t);
+        if (rc == PCC_OK) break;
+        if (rc != -PCC_EAGAIN) return rc;
+        c->engine->wait_free(-1);  // the stall of L139 / Fig 6 when N checkpoints are in flight
+    }
+    cudaSetDevice(c->device);
+    const uint32_t s = ck->t.slot;
+    cudaEventCreateWithFlags(&ck->ev_train, cudaEventDisableTiming);
+    cudaEventCreate(&ck->ev_begin);
+    cudaEventCreate(&ck->ev_packed);
+    cudaEventCreateWithFlags(&ck->ev_final, cudaEventDisableTiming);
+    cudaEventRecord(ck->ev_train, ts);
+    cudaStreamWaitEvent(c->pack_stream, ck->ev_train, 0);
+    cudaEventRecord(ck->ev_begin, c->pack_stream);
+    ck->remaining = (uint32_t)c->n;
+    {
+        std::lock_guard<std::mutex> lk(c->ck_mu);
+        c->ckpts[ck->t.counter] = ck;
+    }
+    ck->state = PCC_ST_PACKING;
+    c->jobs.push(ck);  // the orchestrator follows the launches as they are published
+
+    SnapParams P{};
+    P.rows = c->rows_dev;
+    P.row_begin = c->row_begin_dev;
+    P.chunk_bytes = c->cb();
+    P.tpc = c->geom.tpc;
+    P.tile_crc = c->tile_crc_dev[s];
+    P.tables = c->tables;
+    P.consts = c->consts;
+    cudaError_t e = cudaSuccess;
+    if (c->zerocopy()) {  // Variant A: K1 stores into the registered file mapping over PCIe
+        P.first = 0;
+        P.count = (uint32_t)c->n;
+        P.ring_base = c->map_dev + c->slot_data_off(s);
+        P.ring_head = 0;
+        P.ring_slots = c->n ? c->n : 1;
+        e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas), c->pack_stream);
+        c->launches += c->n ? 1 : 0;
+        cudaEvent_t ev = get_event(c);
+        cudaEventRecord(ev, c->pack_stream);
+        std::lock_guard<std::mutex> lk(ck->mu);
+        ck->launches.push_back({0, (uint32_t)c->n, ev});
+        ck->launched = (uint32_t)c->n;
+    } else {  // Variant B: HBM ring, windowed by ring space
+        {
+            std::lock_guard<std::mutex> lk(c->ring_mu);
+            ck->ring_start = c->ring_head;
+            c->ring_head += c->n;
+        }
+        uint64_t done = 0;
+        while (done < c->n && e == cudaSuccess) {
+            uint64_t k;
+            {
+                std::unique_lock<std::mutex> lk(c->ring_mu);
+                c->ring_cv.wait(lk, [&] { return c->ring_tail + c->ring_slots > ck->ring_start + done; });
+                k = std::min<uint64_t>(c->n - done, c->ring_tail + c->ring_slots - (ck->ring_start + done));
+            }
+            P.first = (uint32_t)done;
+            P.count = (uint32_t)k;
+            P.ring_base = c->ring;
+            P.ring_head = ck->ring_start % c->ring_slots;
+            P.ring_slots = c->ring_slots;
+            e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas), c->pack_stream);
+            c->launches += 1;
+            cudaEvent_t ev = get_event(c);
+            cudaEventRecord(ev, c->pack_stream);
+            {
+                std::lock_guard<std::mutex> lk(ck->mu);
+                ck->launches.push_back({(uint32_t)done, (uint32_t)k, ev});
+                ck->launched = (uint32_t)(done + k);
+            }
+            ck->cv.notify_all();
+            done += k;
+        }
+    }
+    cudaEventRecord(ck->ev_packed, c->pack_stream);
+    cudaEventRecord(c->ev_guard, c->pack_stream);
+    c->guard_armed = true;
+    // chunk CRCs -> slice digest, then the table to pinned host memory for the header
+    cudaMemsetAsync(c->scratch_dev[s], 0, 4 * sizeof(uint32_t), c->pack_stream);
+    FinalizeParams F{};
+    F.tile_crc = c->tile_crc_dev[s];
+    F.n = (uint32_t)c->n;
+    F.tpc = c->geom.tpc;
+    F.tile_shift = c->geom.tile_shift;
+    F.chunk_shift = c->geom.chunk_shift;
+    F.ff = c->geom.ff;
+    F.crc_out = c->crc_dev[s];
+    F.scratch = c->scratch_dev[s];
+    if (e == cudaSuccess) e = launch_finalize(F, c->pack_stream);
+    if (c->n) c->launches += 1;
+    cudaMemcpyAsync(c->crc_dev[s] + c->n, c->scratch_dev[s] + 3, 4, cudaMemcpyDeviceToDevice, c->pack_stream);
+    cudaMemcpyAsync(c->crc_host[s], c->crc_dev[s], (c->n + 1) * sizeof(uint32_t), cudaMemcpyDeviceToHost,
+                    c->pack_stream);
+    cudaEventRecord(ck->ev_final, c->pack_stream);
+    if (e != cudaSuccess) {
+        int rc = cuda_error(e, "K1 launch");
+        fail_ckpt(c, ck, rc);
+        std::lock_guard<std::mutex> lk(ck->mu);
+        ck->launch_failed = true;
+        ck->cv.notify_all();
+    }
+    *out = ck->t.counter;
+    return PCC_OK;
+}
+
+int pcc_guard(pcc_ctx *c, void *train_stream) {
+    if (!c) return set_error(PCC_EINVAL, "ctx");
+    if (!c->guard_armed) return PCC_OK;
+    cudaError_t e = cudaStreamWaitEvent(static_cast<cudaStream_t>(train_stream), c->ev_guard, 0);
+    return e == cudaSuccess ? PCC_OK : cuda_error(e, "guard");
+}
+
+static std::shared_ptr<Ckpt> find_ck(pcc_ctx *c, pcc_handle h) {
+    std::lock_guard<std::mutex> lk(c->ck_mu);
+    auto it = c->ckpts.find(h);
+    return it == c->ckpts.end() ? nullptr : it->second;
+}
+
+static bool terminal(int s) {
+    return s == PCC_ST_LOCAL_COMMIT || s == PCC_ST_GLOBAL_COMMIT || s == PCC_ST_OBSOLETE || s == PCC_ST_FAILED;
+}
+
+int pcc_poll(pcc_ctx *c, pcc_handle h, int *state) {
+    if (!c || !state) return set_error(PCC_EINVAL, "args");
+    auto ck = find_ck(c, h);
+    if (!ck) return set_error(PCC_EINVAL, "unknown handle");
+    int s = ck->state.load();
+    if (s == PCC_ST_PACKING && cudaEventQuery(ck->ev_packed) == cudaSuccess) s = PCC_ST_PACKED;
+    if (s == PCC_ST_LOCAL_COMMIT && c->cfg.world > 1) {
+        uint64_t g = c->engine->global_iter();
+        if (g != UINT64_MAX && g >= ck->t.iter) s = PCC_ST_GLOBAL_COMMIT;
+    }
+    *state = s;
+    return PCC_OK;
+}
+
+int pcc_wait(pcc_ctx *c, pcc_handle h, int64_t timeout_us) {
+    if (!c) return set_error(PCC_EINVAL, "ctx");
+    auto ck = find_ck(c, h);
+    if (!ck) return set_error(PCC_EINVAL, "unknown handle");
+    std::unique_lock<std::mutex> lk(c->ck_mu);
+    auto pred = [&] { return terminal(ck->state.load()); };
+    if (timeout_us < 0)
+        c->ck_cv.wait(lk, pred);
+    else if (!c->ck_cv.wait_for(lk, std::chrono::microseconds(timeout_us), pred))
+        return set_error(PCC_ETIMEDOUT, "wait");
+    if (ck->state.load() == PCC_ST_FAILED) return ck->err.load() ? ck->err.load() : -PCC_EIO;
+    return PCC_OK;
+}
+
+int pcc_drain(pcc_ctx *c, int64_t timeout_us) {
+    if (!c) return set_error(PCC_EINVAL, "ctx");
+    std::unique_lock<std::mutex> lk(c->ck_mu);
+    auto pred = [&] {
+        for (auto &kv : c->ckpts)
+            if (!terminal(kv.second->state.load())) return false;
+        return true;
+    };
+    if (timeout_us < 0)
+        c->ck_cv.wait(lk, pred);
+    else if (!c->ck_cv.wait_for(lk, std::chrono::microseconds(timeout_us), pred))
+        return set_error(PCC_ETIMEDOUT, "drain");
+    return PCC_OK;
+}
+
+// Collective backpressure (SURVEY §7 "hard parts"): a rank without a free slot cannot just
+// block, because only a g-advance frees slots; every rank runs the same rounds of
+// need = MAX(no free slot), g = MIN(L_r) until nobody needs.
+static int dp_backpressure(pcc_ctx *c) {
+    for (int round = 0;; ++round) {
+        int64_t v[2] = {c->engine->has_free() ? 0 : 1, 0};
+        int rc = c->nccl.allreduce_i64(v, 1, NcclComm::kMax, c->red_dev, c->red_host, c->aux_stream);
+        if (rc) return rc;
+        if (v[0] == 0) return PCC_OK;
+        // let local persists progress, then advance g
+        c->engine->wait_free(2000);
+        uint64_t L = c->engine->local_latest();
+        int64_t g[1] = {L == UINT64_MAX ? -1 : (int64_t)L};
+        rc = c->nccl.allreduce_i64(g, 1, NcclComm::kMin, c->red_dev, c->red_host, c->aux_stream);
+        if (rc) return rc;
+        if (g[0] >= 0) c->engine->apply_global((uint64_t)g[0]);
+    }
+}
+
+int pcc_commit(pcc_ctx *c, uint64_t *committed_iter) {
+    if (!c) return set_error(PCC_EINVAL, "ctx");
+    if (!c->registered) return set_error(PCC_ESTATE, "not registered");
+    if (c->cfg.world == 1) {
+        if (committed_iter) *committed_iter = c->engine->local_latest();
+        return PCC_OK;
+    }
+    uint64_t L = c->engine->local_latest();
+    int64_t g[1] = {L == UINT64_MAX ? -1 : (int64_t)L};
+    int rc = c->nccl.allreduce_i64(g, 1, NcclComm::kMin, c->red_dev, c->red_host, c->aux_stream);
+    if (rc) return rc;
+    if (g[0] >= 0) rc = c->engine->apply_global((uint64_t)g[0]);
+    if (committed_iter) *committed_iter = c->engine->global_iter();
+    return rc;
+}
+
+int pcc_info(pcc_ctx *c, pcc_handle h, pcc_ckpt_info *info, uint32_t *crc, uint32_t crc_cap) {
+    if (!c || !info) return set_error(PCC_EINVAL, "args");
+    auto ck = find_ck(c, h);
+    if (!ck) return set_error(PCC_EINVAL, "unknown handle");
+    std::memset(info, 0, sizeof(*info));
+    info->iter = ck->t.iter;
+    info->counter = ck->t.counter;
+    info->slot = ck->t.slot;
+    int st = 0;
+    pcc_poll(c, h, &st);
+    info->state = (uint32_t)st;
+    info->n_chunks = (uint32_t)c->n;
+    info->t_call_us = ck->t_call;
+    if (terminal(ck->state.load()) || ck->state.load() == PCC_ST_PERSISTED) {
+        info->digest = ck->digest;
+        info->t_landed_us = ck->t_landed;
+        info->t_persisted_us = ck->t_persisted;
+        info->t_committed_us = ck->t_committed;
+        info->pack_ms = ck->pack_ms;
+        info->finalize_ms = ck->fin_ms;
+        if (crc)
+            for (uint32_t i = 0; i < crc_cap && i < ck->crc.size(); ++i) crc[i] = ck->crc[i];
+    }
+    return PCC_OK;
+}
+
+int pcc_geometry(pcc_ctx *c, uint64_t *n_chunks, uint64_t *first, uint64_t *count, uint64_t *end_bytes) {
+    if (!c || !c->registered) return set_error(PCC_ESTATE, "not registered");
+    if (n_chunks) *n_chunks = c->layout.C;
+    if (first) *first = c->first;
+    if (count) *count = c->n;
+    if (end_bytes) *end_bytes = c->layout.end;
+    return PCC_OK;
+}
+
+uint64_t pcc_kernel_launches(pcc_ctx *c) { return c ? c->launches.load() : 0; }
+
+int pcc_nccl_unique_id(void *out128) {
+    if (!out128) return set_error(PCC_EINVAL, "out");
+    return pcc_nccl_unique_id_impl(out128);
+}
+
+int pcc_latest(const char *path, uint64_t *global_iter, uint64_t *local_iter) {
+    if (!path) return set_error(PCC_EINVAL, "path");
+    int fd = ::open(path, O_RDONLY);
+    if (fd < 0) return set_error(PCC_ENOENT, "no file");
+    alignas(4096) static thread_local uint8_t buf[kPage];
+    PtrRecord best;
+    for (int k = 0; k < 2; ++k) {
+        if (::pread(fd, buf, kPage, k * kPage) != (ssize_t)kPage) continue;
+        PtrRecord r = decode_ptr(buf);
+        if (r.valid && (!best.valid || r.seq > best.seq)) best = r;
+    }
+    ::close(fd);
+    if (!best.valid) return set_error(PCC_ENOENT, "no valid pointer record");
+    if (global_iter) *global_iter = best.global_iter;
+    if (local_iter) *local_iter = best.local_iter;
+    return PCC_OK;
+}
+
+int pcc_close(pcc_ctx *c) {
+    if (!c) return PCC_OK;
+    pcc_drain(c, -1);
+    c->jobs.close();
+    if (c->orchestrator.joinable()) c->orchestrator.join();
+    c->tasks.close();
+    for (auto &t : c->persisters)
+        if (t.joinable()) t.join();
+    cudaSetDevice(c->device);
+    cudaDeviceSynchronize();
+    {
+        std::lock_guard<std::mutex> lk(c->ck_mu);
+        for (auto &kv : c->ckpts) destroy_ckpt_events(c, kv.second.get());
+        c->ckpts.clear();
+    }
+    free_registration(c);
+    for (auto e : c->evpool) cudaEventDestroy(e);
+    cudaEventDestroy(c->ev_guard);
+    cudaStreamDestroy(c->pack_stream);
+    cudaStreamDestroy(c->copy_stream);
+    cudaStreamDestroy(c->aux_stream);
+    c->nccl.destroy();
+    if (c->red_dev) cudaFree(c->red_dev);
+    if (c->red_host) cudaFreeHost(c->red_host);
+    if (c->fd >= 0) ::close(c->fd);
+    delete c;
+    return PCC_OK;
+}
+
+}  // extern "C"
+
+// ------------------------------------------------------------------------- restore
+namespace {
+
+int pread_full(int fd, char *p, uint64_t n, uint64_t off) {
+    while (n) {
+        ssize_t r = ::pread(fd, p, n, (off_t)off);
+        if (r < 0) {
+            if (errno == EINTR) continue;
+            return set_errno_error("pread chunk", errno);
+        }
+        if (r == 0) return set_error(PCC_EIO, "short read (truncated file)");
+        p += r;
+        n -= (uint64_t)r;
+        off += (uint64_t)r;
+    }
+    return PCC_OK;
+}
+
+struct SlotScan {
+    std::map<uint64_t, uint32_t> complete;  // iter -> slot (COMPLETE, header CRC ok, layout ok)
+    std::map<uint64_t, uint32_t> bad_layout;
+    PtrRecord best;
+};
+
+int scan_file(pcc_ctx *c, SlotScan *S) {
+    uint8_t *buf = static_cast<uint8_t *>(std::aligned_alloc(kPage, header_bytes(c->n)));
+    if (!buf) return set_error(PCC_ENOMEM, "scan buffer");
+    for (int k = 0; k < 2; ++k) {
+        if (::pread(c->fd, buf, kPage, k * kPage) != (ssize_t)kPage) continue;
+        PtrRecord r = decode_ptr(buf);
+        if (r.valid && r.rank == (uint32_t)c->cfg.rank && r.world == (uint32_t)c->cfg.world &&
+            (!S->best.valid || r.seq > S->best.seq))
+            S->best = r;
+    }
+    const uint64_t H = header_bytes(c->n);
+    for (uint32_t s = 0; s < c->n_slots; ++s) {
+        if (::pread(c->fd, buf, H, slot_offset(s, c->n, c->cb())) != (ssize_t)H) continue;
+        HeaderView v = decode_header(buf, c->sgeom, s);
+        if (!v.ok) continue;
+        if (v.layout_ok)
+            S->complete[v.iter] = s;
+        else
+            S->bad_layout[v.iter] = s;
+    }
+    std::free(buf);
+    return PCC_OK;
+}
+
+// K2 over this rank's slice of the checkpoint in `slot`: H2D into the HBM ring, verify every
+// chunk's CRC32C against the header table while scattering into the registered tensors.
+int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
+    const uint64_t n = c->n, cb = c->cb();
+    bad_out->clear();
+    if (n == 0) return PCC_OK;
+    const uint64_t H = header_bytes(n);
+    uint8_t *hdr = static_cast<uint8_t *>(std::aligned_alloc(kPage, H));
+    int rc = pread_full(c->fd, reinterpret_cast<char *>(hdr), H, slot_offset(slot, n, cb));
+    if (rc) {
+        std::free(hdr);
+        return rc;
+    }
+    HeaderView v = decode_header(hdr, c->sgeom, slot);
+    uint32_t *expect = nullptr, *bad = nullptr, *crc = nullptr, *tile = nullptr, *scr = nullptr;
+    cudaError_t e = cudaSuccess;
+    auto done = [&](int r) {
+        cudaFree(expect);
+        cudaFree(bad);
+        cudaFree(crc);
+        cudaFree(tile);
+        cudaFree(scr);
+        std::free(hdr);
+        return r;
+    };
+    if (!v.ok || !v.layout_ok) return done(set_error(PCC_ELAYOUT, "slot header"));
+    if ((e = cudaMalloc(&expect, n * 4)) || (e = cudaMalloc(&bad, n * 4)) || (e = cudaMalloc(&crc, n * 4)) ||
+        (e = cudaMalloc(&tile, n * c->geom.tpc * 4)) || (e = cudaMalloc(&scr, 16)))
+        return done(cuda_error(e, "restore buffers"));
+    cudaMemcpy(expect, v.crc, n * 4, cudaMemcpyHostToDevice);
+    cudaMemset(scr, 0, 16);
+    // ring for restore: zero-copy mode has none; allocate one batch worth
+    char *ring = c->ring;
+    uint64_t R = c->ring_slots;
+    bool own_ring = false;
+    if (!ring) {
+        R = std::min<uint64_t>(n, 16);
+        if ((e = cudaMalloc(&ring, R * cb))) return done(cuda_error(e, "restore ring"));
+        own_ring = true;
+    }
+    SnapParams P{};
+    P.rows = c->rows_dev;
+    P.row_begin = c->row_begin_dev;
+    P.chunk_bytes = cb;
+    P.tpc = c->geom.tpc;
+    P.ring_base = ring;
+    P.ring_slots = R;
+    P.tile_crc = tile;
+    P.tables = c->tables;
+    P.consts = c->consts;
+    cudaEvent_t ev = get_event(c);
+    const uint64_t data0 = c->slot_data_off(slot);
+    for (uint64_t j0 = 0; j0 < n && rc == PCC_OK; j0 += R) {
+        const uint64_t k = std::min<uint64_t>(R, n - j0);
+        for (uint64_t i = 0; i < k && rc == PCC_OK; ++i) {
+            const char *src;
+            if (c->mapfile()) {
+                src = c->map + data0 + (j0 + i) * cb;
+            } else {  // pread into a pinned staging slot, then H2D (the slot is reused after the copy)
+                char *st = c->staging + (i % c->staging_slots) * cb;
+                if (i >= c->staging_slots) cudaStreamSynchronize(c->copy_stream);
+                rc = pread_full(c->fd, st, cb, data0 + (j0 + i) * cb);
+                src = st;
+            }
+            if (rc == PCC_OK) cudaMemcpyAsync(ring + i * cb, src, cb, cudaMemcpyHostToDevice, c->copy_stream);
+        }
+        cudaEventRecord(ev, c->copy_stream);
+        cudaStreamWaitEvent(c->pack_stream, ev, 0);
+        P.first = (uint32_t)j0;
+        P.count = (uint32_t)k;
+        P.ring_head = (R - j0 % R) % R;
+        if ((e = launch_unpack(P, snapshot_grid(c->device, (uint32_t)(k * P.tpc), 0), c->pack_stream)))
+            rc = cuda_error(e, "K2");
+        c->launches += 1;
+        cudaEventRecord(ev, c->pack_stream);
+        cudaStreamWaitEvent(c->copy_stream, ev, 0);  // next batch's H2D after this K2 read the ring
+    }
+    FinalizeParams F{};
+    F.tile_crc = tile;
+    F.n = (uint32_t)n;
+    F.tpc = c->geom.tpc;
+    F.tile_shift = c->geom.tile_shift;
+    F.chunk_shift = c->geom.chunk_shift;
+    F.ff = c->geom.ff;
+    F.crc_out = crc;
+    F.expect = expect;
+    F.bad = bad;
+    F.scratch = scr;
+    if (rc == PCC_OK && (e = launch_finalize(F, c->pack_stream))) rc = cuda_error(e, "finalize");
+    c->launches += 1;
+    std::vector<uint32_t> flags(n);
+    uint32_t sc[4] = {0, 0, 0, 0};
+    if (rc == PCC_OK) {
+        cudaMemcpyAsync(flags.data(), bad, n * 4, cudaMemcpyDeviceToHost, c->pack_stream);
+        cudaMemcpyAsync(sc, scr, 16, cudaMemcpyDeviceToHost, c->pack_stream);
+        if ((e = cudaStreamSynchronize(c->pack_stream))) rc = cuda_error(e, "restore sync");
+    }
+    cudaStreamSynchronize(c->copy_stream);
+    put_event(c, ev);
+    if (own_ring) cudaFree(ring);
+    if (rc) return done(rc);
+    for (uint64_t j = 0; j < n; ++j)
+        if (flags[j]) bad_out->push_back((uint32_t)(c->first + j));
+    if (!bad_out->empty()) return done(set_error(PCC_ECORRUPT, "chunk CRC32C mismatch"));
+    if (sc[3] != v.digest) return done(set_error(PCC_ECORRUPT, "slice digest mismatch"));
+    return done(PCC_OK);
+}
+
+int restore_dp(pcc_ctx *c, SlotScan *S, uint64_t want_iter, uint32_t flags, uint64_t *restored_iter,
+               uint32_t *bad_chunks, uint32_t bad_cap, uint32_t *n_bad) {
+    (void)S; (void)want_iter; (void)flags; (void)restored_iter; (void)bad_chunks; (void)bad_cap; (void)n_bad;
+    return set_error(PCC_ESTATE, "world > 1 restore not built yet");
+}
+
+}  // namespace
+
+extern "C" int pcc_restore(pcc_ctx *c, uint64_t want_iter, uint32_t flags, uint64_t *restored_iter,
+                           uint32_t *bad_chunks, uint32_t bad_cap, uint32_t *n_bad) {
+    if (!c) return set_error(PCC_EINVAL, "ctx");
+    if (!c->registered) return set_error(PCC_ESTATE, "not registered");
+    if (n_bad) *n_bad = 0;
+    if (c->fd < 0) return set_error(PCC_ENOENT, "no file (NULLSINK)");
+    pcc_drain(c, -1);
+    cudaSetDevice(c->device);
+    SlotScan S;
+    int rc = scan_file(c, &S);
+    if (rc) return rc;
+    if (c->cfg.world > 1) return restore_dp(c, &S, want_iter, flags, restored_iter, bad_chunks, bad_cap, n_bad);
+    uint64_t target = want_iter;
+    if (target == PCC_LATEST) {
+        if (!S.best.valid) return set_error(PCC_ENOENT, "no valid pointer record");
+        target = S.best.global_iter;
+    }
+    int first_rc = 0;
+    bool reported = false;
+    for (;;) {
+        int cand;
+        std::vector<uint32_t> bad;
+        auto it = S.complete.find(target);
+        if (it == S.complete.end()) {
+            cand = S.bad_layout.count(target) ? set_error(PCC_ELAYOUT, "registration differs from checkpoint")
+                                               : set_error(PCC_ENOENT, "iter not held");
+        } else {
+            cand = verify_scatter(c, it->second, &bad);
+        }
+        if (cand == PCC_OK) {
+            if (restored_iter) *restored_iter = target;
+            return PCC_OK;
+        }
+        if (!reported) {
+            reported = true;
+            first_rc = cand;
+            if (n_bad) *n_bad = (uint32_t)bad.size();
+            for (size_t i = 0; i < bad.size() && i < bad_cap && bad_chunks; ++i) bad_chunks[i] = bad[i];
+        }
+        if (!(flags & PCC_FALLBACK)) return first_rc;
+        auto lower = S.complete.lower_bound(target);  // first >= target
+        if (lower == S.complete.begin()) return first_rc;
+        --lower;
+        target = lower->first;
+    }
+}

@@ -1,0 +1,169 @@
+"""The full path through pccheck.h on one B200: checkpoint -> copy -> persist -> commit ->
+restore, checked against the oracle byte for byte on the files the library wrote."""
+import os
+import struct
+
+import numpy as np
+import pytest
+
+import oracle
+from synth import config_tensors, make_state, perturb_state, host_bytes
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def pcc():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import paper_conf_asplos_strati0k25_b200 as p
+    return p
+
+
+@pytest.fixture
+def shm(tmp_path):
+    d = "/dev/shm" if os.path.isdir("/dev/shm") else str(tmp_path)
+    p = os.path.join(d, f"pcc_test_{os.getpid()}_{np.random.randint(1 << 30)}.pcc")
+    yield p
+    if os.path.exists(p):
+        os.unlink(p)
+
+
+MODES = {
+    "mapfile": lambda p: p.MAPFILE,
+    "mapfile_zerocopy": lambda p: p.MAPFILE | p.ZEROCOPY,
+    "pwrite_odirect": lambda p: p.ODIRECT | p.FSYNC,
+    "pwrite_small_ring": lambda p: p.ODIRECT,
+}
+
+
+def _file_slice_image(path, slot, n, cb):
+    with open(path, "rb") as f:
+        f.seek(oracle.slot_offset(slot, n, cb) + oracle.header_bytes(n))
+        return np.frombuffer(f.read(n * cb), dtype=np.uint8)
+
+
+def _check_file_against_oracle(path, specs, ts, cb, info, n_slots):
+    hb = [host_bytes(t) for t in ts]
+    nbytes = [s.nbytes for s in specs]
+    dt = [s.code for s in specs]
+    img = oracle.pack(hb, 256, cb)
+    c = img.nbytes // cb
+    crcs = [int(x) for x in oracle.chunk_crcs(img, cb)]
+    # data region
+    got = _file_slice_image(path, info["slot"], c, cb)
+    assert np.array_equal(got, img)
+    # slot header: byte-identical to the oracle's O5 encoding
+    exp_hdr = oracle.slot_header(2, info["iter"], info["counter"], cb, 0, 1, c, 0, c, len(specs), 256,
+                                 oracle.layout_crc(nbytes, dt, 256, cb), oracle.crc32c(img), info["slot"], crcs)
+    with open(path, "rb") as f:
+        f.seek(oracle.slot_offset(info["slot"], c, cb))
+        assert f.read(len(exp_hdr)) == exp_hdr
+    # the oracle restores what the library wrote
+    rc, it, bad, outs = oracle.restore([path], n_slots, nbytes, dt, 256, cb)
+    assert rc == 0 and it == info["iter"] and bad == []
+    assert all(np.array_equal(o, h) for o, h in zip(outs, hb))
+
+
+@pytest.mark.parametrize("mode", sorted(MODES))
+def test_checkpoint_file_matches_oracle(pcc, shm, mode):
+    specs = config_tensors("c1")
+    cb = 4 << 20
+    ts = make_state(specs, "cuda", seed=1, it=0)
+    ring = (3 * cb) if mode == "pwrite_small_ring" else 0
+    with pcc.PCCheck(shm, chunk_bytes=cb, max_inflight=2, flags=MODES[mode](pcc), ring_bytes=ring,
+                     staging_bytes=4 * cb) as ck:
+        ck.register(ts)
+        for it in (10, 20, 30):
+            perturb_state(ts, specs, seed=1, it=it)
+            h = ck.checkpoint(it)
+            ck.guard()
+            ck.wait(h)
+            info = ck.info(h, with_crc=True)
+            assert info["state_name"] == "LOCAL_COMMIT"
+            _check_file_against_oracle(shm, specs, ts, cb, info, 3)
+        assert pcc.latest(shm) == (30, 30)
+
+
+def test_n_in_flight_and_guard(pcc, shm):
+    """N=3 checkpoints issued back to back while the 'optimizer' rewrites the state after
+    each guard: every checkpoint must hold the state as it was at its own call (L139)."""
+    specs = config_tensors("c1")
+    cb = 4 << 20
+    ts = make_state(specs, "cuda", seed=3, it=0)
+    expected = {}
+    with pcc.PCCheck(shm, chunk_bytes=cb, max_inflight=3, flags=pcc.MAPFILE, ring_bytes=40 * cb) as ck:
+        ck.register(ts)
+        hs = []
+        for it in range(10, 60, 10):
+            perturb_state(ts, specs, seed=3, it=it)
+            torch.cuda.synchronize()
+            expected[it] = oracle.pack([host_bytes(t) for t in ts], 256, cb)
+            hs.append(ck.checkpoint(it))
+            ck.guard()  # U-gate before the next update
+        for h in hs:
+            ck.wait(h)
+        states = [ck.info(h)["state_name"] for h in hs]
+        assert all(s in ("LOCAL_COMMIT", "OBSOLETE") for s in states)
+        assert states[-1] == "LOCAL_COMMIT"
+        for h in hs:
+            inf = ck.info(h, with_crc=True)
+            if inf["state_name"] == "LOCAL_COMMIT":
+                assert inf["crc"] == [int(x) for x in oracle.chunk_crcs(expected[inf["iter"]], cb)]
+        assert pcc.latest(shm)[0] == 50
+        rc, it, bad, outs = oracle.restore([shm], 4, [s.nbytes for s in specs], [s.code for s in specs], 256, cb)
+        assert rc == 0 and it == 50
+        assert np.array_equal(np.concatenate(outs), np.concatenate(
+            [expected[50][o:o + s.nbytes] for o, s in zip(oracle.layout([s.nbytes for s in specs], 256, cb)[0], specs)]))
+
+
+@pytest.mark.parametrize("mode", ["mapfile", "pwrite_odirect"])
+def test_restore_roundtrip_and_faults(pcc, shm, mode):
+    specs = config_tensors("c1")
+    cb = 4 << 20
+    ts = make_state(specs, "cuda", seed=5, it=0)
+    with pcc.PCCheck(shm, chunk_bytes=cb, max_inflight=2, flags=MODES[mode](pcc)) as ck:
+        ck.register(ts)
+        perturb_state(ts, specs, 5, 10)
+        ck.wait(ck.checkpoint(10))
+        s10 = [host_bytes(t).copy() for t in ts]
+        perturb_state(ts, specs, 5, 20)
+        h20 = ck.checkpoint(20)
+        ck.wait(h20)
+        s20 = [host_bytes(t).copy() for t in ts]
+        perturb_state(ts, specs, 5, 99)  # training moves on, then we crash and restore
+        it, bad = ck.restore()
+        assert it == 20 and bad == []
+        assert all(np.array_equal(host_bytes(t), s) for t, s in zip(ts, s20))
+        # corrupt chunk 3 of iter 20's slot: one bit
+        inf = ck.info(h20)
+        c = ck.geometry()["count"]
+        off = oracle.slot_offset(inf["slot"], c, cb) + oracle.header_bytes(c) + 3 * cb + 777
+        with open(shm, "r+b") as f:
+            f.seek(off)
+            b = f.read(1)
+            f.seek(off)
+            f.write(bytes([b[0] ^ 0x04]))
+        with pytest.raises(pcc.PCCError) as ei:
+            ck.restore()
+        assert ei.value.code == pcc.ECORRUPT and ei.value.bad_chunks == [3]
+        it, bad = ck.restore(fallback=True)
+        assert it == 10
+        assert all(np.array_equal(host_bytes(t), s) for t, s in zip(ts, s10))
+
+
+def test_nullsink_and_launch_count(pcc):
+    specs = config_tensors("c2")
+    ts = make_state(specs, "cuda", seed=0, it=0)
+    with pcc.PCCheck(None, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.NULLSINK) as ck:
+        ck.register(ts)
+        before = ck.kernel_launches()
+        for it in range(1, 4):
+            ck.wait(ck.checkpoint(it))
+        assert ck.kernel_launches() - before == 3 * 2  # K1 + finalize per checkpoint
+        h = ck.checkpoint(4)
+        ck.wait(h)
+        inf = ck.info(h)
+        img = oracle.pack([host_bytes(t) for t in ts], 256, 64 << 20)
+        assert inf["digest"] == oracle.crc32c(img)

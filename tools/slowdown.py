@@ -1,0 +1,93 @@
+"""Training-iteration slowdown with a checkpoint every `every` iterations vs none
+(BASELINE.json metric, second half).
+
+Random-init torchvision VGG-16, fp32, SGD(momentum=0.9), batch 32 of random 3x224x224
+images with random labels (PAPER Table 3: VGG16, batch 32).  The checkpointed state
+is every parameter and its momentum buffer (R11).  Per iteration: forward + backward, then
+pcc_guard (the U-gate of L139: the update must not overwrite the state K1 is still
+reading), then optimizer.step(); after the step of every `every`-th iteration,
+pcc_checkpoint(iter).  Both runs use the same model, inputs and iteration count; time is
+measured with CUDA events around the whole loop.
+"""
+from __future__ import annotations
+
+import os
+import statistics
+
+
+def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=None):
+    import torch
+    import torchvision
+
+    torch.manual_seed(0)
+    dev = torch.device("cuda")
+    model = torchvision.models.vgg16(weights=None).to(dev)
+    opt = torch.optim.SGD(model.parameters(), lr=1e-3, momentum=0.9)
+    x = torch.randn(batch, 3, 224, 224, device=dev)
+    y = torch.randint(0, 1000, (batch,), device=dev)
+    lossf = torch.nn.CrossEntropyLoss()
+    stream = torch.cuda.current_stream()
+
+    def step():
+        opt.zero_grad(set_to_none=True)
+        lossf(model(x), y).backward()
+
+    for _ in range(2):  # momentum buffers exist after the first step
+        step()
+        opt.step()
+    state = []
+    for p in model.parameters():
+        state += [p.data, opt.state[p]["momentum_buffer"]]
+    shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
+    path = path or os.path.join(shm, f"pcc_slowdown_{os.getpid()}.pcc")
+    ck = pcc.PCCheck(path, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.MAPFILE)
+    ck.register(state)
+
+    def loop(n, checkpoint, it0):
+        handles = []
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        per = []
+        e0.record(stream)
+        last = e0
+        for i in range(1, n + 1):
+            step()
+            if checkpoint:
+                ck.guard(stream)
+            opt.step()
+            if checkpoint and i % every == 0:
+                handles.append(ck.checkpoint(it0 + i, stream))
+            ev = torch.cuda.Event(enable_timing=True)
+            ev.record(stream)
+            per.append((last, ev))
+            last = ev
+        e1.record(stream)
+        e1.synchronize()
+        total = e0.elapsed_time(e1)
+        for h in handles:
+            ck.wait(h)
+        its = sorted(a.elapsed_time(b) for a, b in per)
+        return total, its
+
+    loop(warmup, False, 0)
+    base_t, ck_t, its_b, its_c = [], [], [], []
+    it0 = 1000
+    for r in range(runs):
+        t, its = loop(iters, False, 0)
+        base_t.append(t)
+        its_b += its
+        t, its = loop(iters, True, it0)
+        it0 += 1000
+        ck_t.append(t)
+        its_c += its
+    ck.drain()
+    ck.close()
+    if os.path.exists(path):
+        os.unlink(path)
+    b, c = statistics.mean(base_t), statistics.mean(ck_t)
+    pct = lambda v, q: sorted(v)[min(len(v) - 1, int(q * len(v)))]  # noqa: E731
+    return {"model": "vgg16 fp32 SGD(momentum) batch 32, random init, synthetic inputs",
+            "every": every, "iters": iters, "runs": runs,
+            "iter_ms_no_ckpt": b / iters, "iter_ms_ckpt": c / iters,
+            "slowdown_pct": (c / b - 1.0) * 100.0,
+            "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
+            "state_bytes": sum(t.numel() * t.element_size() for t in state)}
