@@ -61,7 +61,7 @@ class ClockSampler:
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}",
-                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -162,7 +162,7 @@ def run_reference(args, rank, world):
           for t in state]
     nb = [s.nbytes for s in specs]
     off, end, c = O.layout(nb, 256, cb)
-    per_step = max(1, min(c, 2))
+    per_step = 1
     times = []
     j = 0
     for step in range(args.warmup + args.steps):
@@ -191,11 +191,12 @@ def run_reference(args, rank, world):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=30)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="c2")
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
     ap.add_argument("--inflight", type=int, default=2)
+    ap.add_argument("--ring-slices", type=int, default=2, help="HBM ring = this many slices")
     ap.add_argument("--no-slowdown", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--mode", default="mapfile", choices=["mapfile", "zerocopy", "nullsink", "pwrite"])
@@ -225,12 +226,15 @@ def main():
         obj = [pcc.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
+    from paper_conf_asplos_strati0k25_b200 import k_layout
+    n_est = k_layout([(1 << 20, s.nbytes, s.code) for s in specs], 256, cb)[2]
+    slice_est = -(-n_est // world) * cb
     flags = {"mapfile": pcc.MAPFILE, "zerocopy": pcc.MAPFILE | pcc.ZEROCOPY, "nullsink": pcc.NULLSINK,
              "pwrite": pcc.ODIRECT}[args.mode]
     shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
     path = None if args.mode == "nullsink" else os.path.join(shm, f"pcc_bench_{os.getpid()}_r{rank}.pcc")
     ck = pcc.PCCheck(path, chunk_bytes=cb, max_inflight=args.inflight, flags=flags, device=local, rank=rank,
-                     world=world, nccl_unique_id=uid, staging_bytes=8 * cb)
+                     world=world, nccl_unique_id=uid, staging_bytes=8 * cb, ring_bytes=args.ring_slices * slice_est)
     ck.register(state)
     geo = ck.geometry()
     slice_bytes = geo["count"] * cb
@@ -344,7 +348,7 @@ def main():
             "data": "synthetic (seeded bit patterns; shapes of the model's params + optimizer state)",
             "config": {"workload": WORKLOADS.get(args.config, args.config), "config": args.config,
                        "state_bytes": state_bytes, "chunk_bytes": cb, "chunks": geo["n_chunks"],
-                       "inflight": args.inflight, "mode": args.mode, "parallelism": f"dp{world}",
+                       "inflight": args.inflight, "mode": args.mode, "hbm_ring_slices": args.ring_slices, "parallelism": f"dp{world}",
                        "target": "DRAM file on /dev/shm (tmpfs), mmap + cudaHostRegister" if args.mode != "nullsink"
                        else "null sink", "l2": "inputs larger than L2 (state >> 126 MB)"},
             "per_gpu_gbs": value / world,

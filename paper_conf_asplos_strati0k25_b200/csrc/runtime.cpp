@@ -578,7 +578,7 @@ int pcc_register(pcc_ctx *c, const pcc_tensor *t, uint32_t nt) {
     if (!c->zerocopy()) {
         uint64_t r = c->cfg.ring_bytes ? c->cfg.ring_bytes / c->cb() : c->n;
         if (r == 0) r = 1;
-        if (r > nn) r = nn;
+        if (r > 8 * nn) r = 8 * nn;  // more than 8 slices of ring cannot be used (N in flight)
         c->ring_slots = r;
         if ((e = cudaMalloc(&c->ring, r * c->cb())) != cudaSuccess) return cuda_error(e, "HBM ring");
         c->ring_done.assign(r, 0);
@@ -669,7 +669,6 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
     cudaEventCreateWithFlags(&ck->ev_final, cudaEventDisableTiming);
     cudaEventRecord(ck->ev_train, ts);
     cudaStreamWaitEvent(c->pack_stream, ck->ev_train, 0);
-    cudaEventRecord(ck->ev_begin, c->pack_stream);
     ck->remaining = (uint32_t)c->n;
     {
         std::lock_guard<std::mutex> lk(c->ck_mu);
@@ -693,6 +692,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
         P.ring_base = c->map_dev + c->slot_data_off(s);
         P.ring_head = 0;
         P.ring_slots = c->n ? c->n : 1;
+        cudaEventRecord(ck->ev_begin, c->pack_stream);
         e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas), c->pack_stream);
         c->launches += c->n ? 1 : 0;
         cudaEvent_t ev = get_event(c);
@@ -719,6 +719,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
             P.ring_base = c->ring;
             P.ring_head = ck->ring_start % c->ring_slots;
             P.ring_slots = c->ring_slots;
+            if (done == 0) cudaEventRecord(ck->ev_begin, c->pack_stream);  // K1 time excludes ring waits
             e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas), c->pack_stream);
             c->launches += 1;
             cudaEvent_t ev = get_event(c);
@@ -732,6 +733,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
             done += k;
         }
     }
+    if (c->n == 0) cudaEventRecord(ck->ev_begin, c->pack_stream);
     cudaEventRecord(ck->ev_packed, c->pack_stream);
     cudaEventRecord(c->ev_guard, c->pack_stream);
     c->guard_armed = true;
