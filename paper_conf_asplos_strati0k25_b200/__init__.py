@@ -12,7 +12,7 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libpccheck.so")
+LIB_PATH = os.environ.get("PCC_LIB") or os.path.join(_HERE, "libpccheck.so")  # PCC_LIB: dev A/B builds
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is missing: run `make` (or __graft_entry__.build()) first; "

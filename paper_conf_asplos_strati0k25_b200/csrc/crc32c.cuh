@@ -57,46 +57,92 @@ __host__ __device__ inline uint32_t x8n(const uint32_t *x2n, uint64_t n) {
 }
 
 // ---------------------------------------------------------------- kernel geometry
-// One CTA = 8 warps.  Lane-strided layout: in round r, lane l owns the 16-byte word at
-// warp_base + r*512 + 16*l, so every warp load / store is a contiguous 512 B.  A lane's
-// register is advanced by the 496 zero bytes between its words (gap table G) and then
-// absorbs its word with slicing-by-16 (tables T).  Lanes combine with a 5-level shuffle
-// tree (tables L[k] shift by 16*2^k bytes), warps with x8n constants, tiles and chunks in
-// the finalize kernel.
-constexpr int kWarps = 8;
+// One CTA of 32 warps per SM (all warps share one 96 KiB copy of the tables), tile = 256 KiB
+// of one chunk, warp region = 8 KiB = 16 rounds of 512 B.  In round r lane l owns the
+// 16-byte word at warp_base + r*512 + 16*l, so every warp access is 512 contiguous bytes.
+// Loads go global -> shared with cp.async into a per-warp ring of kStages rounds (each lane
+// only ever reads back its own 16-byte slot, so no barrier is needed), keeping
+// 32 warps x 6 x 512 B = 96 KiB per SM in flight without spending registers.
+// Per round a lane's register becomes  s <- shift(s, 512) ^ raw16(w);  after the last
+// round its contribution is shifted to the warp-region end (shift by 16*(31-l)) and
+// XOR-reduced over the warp, giving the sub-tile CRC; the finalize kernel folds sub-tiles,
+// chunks and the slice digest.
+//
+// Lookups are NIBBLE tables replicated once per lane: entry (table t, nibble v) of lane l
+// sits at word (t*16 + v)*32 + l, i.e. always in bank l.  Every shared load of the CRC is
+// therefore conflict-free (1 wavefront), at 2 lookups per byte.  (Byte-indexed slicing-by-16
+// tables cost 1.25 lookups per byte but random indices collide in banks ~2.9-way on average;
+// ncu showed the L1/shared pipe at 81% with that design, K1 at 0.45 of HBM.)
+constexpr int kWarps = 32;
 constexpr int kThreads = kWarps * 32;
-constexpr int kRounds = 8;                       // rounds per warp per tile
-constexpr uint32_t kRound = 512;                 // bytes per warp per round
-constexpr uint32_t kWarpBytes = kRounds * kRound;  // 4 KiB per warp
-constexpr uint32_t kTile = kWarps * kWarpBytes;    // 32 KiB per CTA tile
-constexpr uint32_t kGap = kRound - 16;             // zero bytes between a lane's words
+constexpr int kRounds = 16;                        // rounds per warp per tile
+constexpr int kStages = 6;                         // cp.async ring depth per warp (rounds in flight)
+constexpr uint32_t kRound = 512;                   // bytes per warp per round
+constexpr uint32_t kWarpBytes = kRounds * kRound;  // 8 KiB per warp
+constexpr uint32_t kTile = kWarps * kWarpBytes;    // 256 KiB per CTA tile
+constexpr uint32_t kStageBytes = kWarps * kStages * kRound;  // 96 KiB of shared staging per CTA
+constexpr int kMaxTileRows = 512;                  // segment rows staged per tile (more -> read from global)
 
-// Shared-memory table block (40 KiB): slicing-by-16, gap shift, 5 tree-level shifts.
+// Shared-memory table block (96 KiB), per-lane replicated nibble tables.
 struct CrcTables {
-    uint32_t T[16][256];     // T[k][b] = raw(b followed by k zero bytes)
-    uint32_t G[4][256];      // G[i][b] = shift(b << 8i, kGap): the zero bytes before a lane's next word
-    uint32_t L[5][4][256];   // L[k][i][b] = shift(b << 8i, 16 << k)
+    uint32_t NT[32][16][32];  // NT[q][v][l] = raw16(16-byte word whose nibble q is v, others 0)
+    uint32_t NF[8][16][32];   // NF[q][v][l] = shift(v << 4q, 512): one round
+    uint32_t NL[8][16][32];   // NL[q][v][l] = shift(v << 4q, 16*(31-l)): lane -> warp-region end
 };
-static_assert(sizeof(CrcTables) == 40 * 1024, "table block size");
+static_assert(sizeof(CrcTables) == 96 * 1024, "table block size");
 
 // Constants that do not need a table.
 struct CrcConsts {
     uint32_t x2n[kX2n];
     uint32_t warp_shift[kWarps];  // x8n((kWarps-1-w) * kWarpBytes)
-    uint32_t x8n_stride_gap;      // x8n(kThreads*16 - 16): generic (ragged-tile) path, zeros between a thread's words
+    uint32_t x8n_stride;          // x8n(kThreads*16): generic (ragged-tile) path, one thread stride
 };
 
-__device__ __forceinline__ uint32_t shift4(const uint32_t (*S)[256], uint32_t v) {
-    return S[0][v & 0xFF] ^ S[1][(v >> 8) & 0xFF] ^ S[2][(v >> 16) & 0xFF] ^ S[3][v >> 24];
+// XOR of the 8 nibble-table entries selected by the nibbles of x.  `tab` = byte address of
+// table t0 (a shared-memory constant), lane4 = lane*4; entry (t0+k, v) of this lane lives at
+// tab + k*2048 + v*128 + lane4.  ((x >> 4k) & 15) << 7 == (x >> (4k-7)) & 0x780.
+// x >> k as IMAD.HI on the FMA pipe (a plain >> becomes SHF on the ALU pipe, which the
+// LOP3s of the lookups already saturate); mul.hi by a power of two is not strength-reduced.
+__device__ __forceinline__ uint32_t shr_fma(uint32_t x, uint32_t pow2) {
+    uint32_t r;
+    asm("mul.hi.u32 %0, %1, %2;" : "=r"(r) : "r"(x), "r"(pow2));
+    return r;
 }
 
-// register s absorbs the 16 bytes w (little-endian words): slicing-by-16.
-__device__ __forceinline__ uint32_t update16(const uint32_t (*T)[256], uint32_t s, uint4 w) {
-    uint32_t x = w.x ^ s;
-    return T[15][x & 0xFF] ^ T[14][(x >> 8) & 0xFF] ^ T[13][(x >> 16) & 0xFF] ^ T[12][x >> 24] ^
-           T[11][w.y & 0xFF] ^ T[10][(w.y >> 8) & 0xFF] ^ T[9][(w.y >> 16) & 0xFF] ^ T[8][w.y >> 24] ^
-           T[7][w.z & 0xFF] ^ T[6][(w.z >> 8) & 0xFF] ^ T[5][(w.z >> 16) & 0xFF] ^ T[4][w.z >> 24] ^
-           T[3][w.w & 0xFF] ^ T[2][(w.w >> 8) & 0xFF] ^ T[1][(w.w >> 16) & 0xFF] ^ T[0][w.w >> 24];
+// (a & 0x780) | lane4 as ONE opaque LOP3: written in C the compiler re-associates it into an
+// AND plus an IADD of a hoisted (table base + lane4) register — one extra instruction per
+// lookup; kept opaque, the table base folds into the LDS's uniform-register + immediate.
+__device__ __forceinline__ uint32_t nib_off(uint32_t a, uint32_t lane4) {
+    uint32_t r;
+    asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(r) : "r"(a), "r"(0x780u), "r"(lane4));
+    return r;
+}
+
+__device__ __forceinline__ uint32_t nib8(const char *tab, uint32_t lane4, uint32_t x) {
+    const uint32_t o0 = nib_off(x * 128u, lane4);                 // nibble 0: << 7
+    const uint32_t o1 = nib_off(x * 8u, lane4);                   // nibble 1: << 3
+    const uint32_t o2 = nib_off(shr_fma(x, 1u << 31), lane4);     // nibble k: >> (4k-7)
+    const uint32_t o3 = nib_off(shr_fma(x, 1u << 27), lane4);
+    const uint32_t o4 = nib_off(shr_fma(x, 1u << 23), lane4);
+    const uint32_t o5 = nib_off(shr_fma(x, 1u << 19), lane4);
+    const uint32_t o6 = nib_off(shr_fma(x, 1u << 15), lane4);
+    const uint32_t o7 = nib_off(shr_fma(x, 1u << 11), lane4);
+    const uint32_t a = *reinterpret_cast<const uint32_t *>(tab + 0 * 2048 + o0) ^
+                       *reinterpret_cast<const uint32_t *>(tab + 1 * 2048 + o1) ^
+                       *reinterpret_cast<const uint32_t *>(tab + 2 * 2048 + o2);
+    const uint32_t b = *reinterpret_cast<const uint32_t *>(tab + 3 * 2048 + o3) ^
+                       *reinterpret_cast<const uint32_t *>(tab + 4 * 2048 + o4) ^
+                       *reinterpret_cast<const uint32_t *>(tab + 5 * 2048 + o5);
+    const uint32_t c = *reinterpret_cast<const uint32_t *>(tab + 6 * 2048 + o6) ^
+                       *reinterpret_cast<const uint32_t *>(tab + 7 * 2048 + o7);
+    return a ^ b ^ c;
+}
+
+// raw16(w): CRC register of the 16 bytes w fed into a zero register (32 nibble lookups).
+__device__ __forceinline__ uint32_t raw16(const CrcTables &tb, uint32_t lane4, uint4 w) {
+    const char *t = reinterpret_cast<const char *>(&tb.NT[0][0][0]);
+    return nib8(t, lane4, w.x) ^ nib8(t + 8 * 2048, lane4, w.y) ^ nib8(t + 16 * 2048, lane4, w.z) ^
+           nib8(t + 24 * 2048, lane4, w.w);
 }
 
 }  // namespace pcc

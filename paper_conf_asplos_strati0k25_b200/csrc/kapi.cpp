@@ -19,6 +19,7 @@ namespace {
 struct Scratch {
     SegRow *rows = nullptr;
     uint32_t *row_begin = nullptr, *tile_crc = nullptr, *scratch = nullptr, *crc_tmp = nullptr;
+    uint2 *tile_rows = nullptr;
     DevGeometry geom;
     ~Scratch() {
         cudaFree(rows);
@@ -26,6 +27,7 @@ struct Scratch {
         cudaFree(tile_crc);
         cudaFree(scratch);
         cudaFree(crc_tmp);
+        cudaFree(tile_rows);
         free_geometry(&geom);
     }
 };
@@ -36,6 +38,7 @@ int prepare(const pcc_tensor *t, uint32_t n, uint32_t align, uint64_t cb, uint64
     int rc = build_layout(t, n, align ? align : 256, cb, first, (int64_t)count, L);
     if (rc) return set_error(PCC_EINVAL, "bad geometry");
     if (first + count > L->C) return set_error(PCC_EINVAL, "chunk range beyond the image");
+    build_tile_rows(L, cb, kTile);
     cudaError_t e;
     int dev = 0;
     cudaGetDevice(&dev);
@@ -46,8 +49,12 @@ int prepare(const pcc_tensor *t, uint32_t n, uint32_t align, uint64_t cb, uint64
     const size_t nrows = L->rows.size() ? L->rows.size() : 1;
     if ((e = cudaMalloc(&S->rows, nrows * sizeof(SegRow))) != cudaSuccess) return cuda_error(e, "rows");
     if ((e = cudaMalloc(&S->row_begin, (count + 1) * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "rb");
-    if ((e = cudaMalloc(&S->tile_crc, count * S->geom.tpc * sizeof(uint32_t))) != cudaSuccess)
+    if ((e = cudaMalloc(&S->tile_crc, count * S->geom.tpc * kWarps * sizeof(uint32_t))) != cudaSuccess)
         return cuda_error(e, "tile crc");
+    if ((e = cudaMalloc(&S->tile_rows, L->tile_rows.size() * sizeof(uint32_t))) != cudaSuccess)
+        return cuda_error(e, "tile rows");
+    cudaMemcpyAsync(S->tile_rows, L->tile_rows.data(), L->tile_rows.size() * sizeof(uint32_t), cudaMemcpyHostToDevice,
+                    s);
     if ((e = cudaMalloc(&S->scratch, 4 * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "scratch");
     if (!L->rows.empty())
         cudaMemcpyAsync(S->rows, L->rows.data(), L->rows.size() * sizeof(SegRow), cudaMemcpyHostToDevice, s);
@@ -57,6 +64,7 @@ int prepare(const pcc_tensor *t, uint32_t n, uint32_t align, uint64_t cb, uint64
     if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_error(e, "upload");
     P->rows = S->rows;
     P->row_begin = S->row_begin;
+    P->tile_rows = S->tile_rows;
     P->chunk_bytes = cb;
     P->first = 0;
     P->count = (uint32_t)count;

@@ -28,38 +28,59 @@
 namespace pcc {
 
 // ------------------------------------------------------------------ table builders
+// raw CRC register of `val` at byte position `pos` of a 16-byte word (followed by 15-pos
+// zero bytes), from the byte-wise table T0.
+__device__ uint32_t raw_byte_at(const uint32_t *T0, uint32_t val, int pos) {
+    uint32_t r = T0[val & 0xFF];
+    for (int z = 0; z < 15 - pos; ++z) r = (r >> 8) ^ T0[r & 0xFF];
+    return r;
+}
+
 __global__ void k_build_tables(CrcTables *tb, CrcConsts *cs) {
     __shared__ uint32_t x2n[kX2n];
-    const int b = threadIdx.x;  // 256 threads
-    if (b == 0) make_x2n(x2n);
-    // T[0]: the byte-wise table, T[k]: byte followed by k zero bytes
-    uint32_t r = b;
+    __shared__ uint32_t T0[256];
+    __shared__ uint32_t vals[48][16];  // distinct entries: NT 32 tables, NF 8, then NL per lane
+    const int t = threadIdx.x;  // 256 threads
+    if (t == 0) make_x2n(x2n);
+    uint32_t r = t;
     for (int k = 0; k < 8; ++k) r = (r & 1u) ? (r >> 1) ^ kPoly : (r >> 1);
-    tb->T[0][b] = r;
+    T0[t] = r;
     __syncthreads();
-    __threadfence_block();
-    for (int k = 1; k < 16; ++k) {
-        uint32_t v = tb->T[k - 1][b];
-        v = (v >> 8) ^ tb->T[0][v & 0xFF];
-        tb->T[k][b] = v;
-        __syncthreads();
+    // NT: 32 nibble positions x 16 values
+    for (int e = t; e < 32 * 16; e += blockDim.x) {
+        const int q = e >> 4, v = e & 15;
+        vals[q][v] = raw_byte_at(T0, (q & 1) ? (v << 4) : v, q >> 1);
     }
-    const uint32_t g = x8n(x2n, kGap);
-    for (int i = 0; i < 4; ++i) tb->G[i][b] = multmodp(g, (uint32_t)b << (8 * i));
-    for (int k = 0; k < 5; ++k) {
-        const uint32_t m = x8n(x2n, 16u << k);
-        for (int i = 0; i < 4; ++i) tb->L[k][i][b] = multmodp(m, (uint32_t)b << (8 * i));
+    // NF: shift by one round
+    const uint32_t xr = x8n(x2n, kRound);
+    if (t < 8 * 16) {
+        const int q = t >> 4, v = t & 15;
+        vals[32 + q][v] = multmodp(xr, (uint32_t)v << (4 * q));
     }
-    if (b < kX2n) cs->x2n[b] = x2n[b];
-    if (b < kWarps) cs->warp_shift[b] = x8n(x2n, (uint64_t)(kWarps - 1 - b) * kWarpBytes);
-    if (b == 0) cs->x8n_stride_gap = x8n(x2n, (uint64_t)kThreads * 16 - 16);
+    __syncthreads();
+    for (int e = t; e < 40 * 16 * 32; e += blockDim.x) {
+        const int tab = e / 512, v = (e >> 5) & 15, l = e & 31;
+        const uint32_t x = vals[tab][v];
+        if (tab < 32)
+            tb->NT[tab][v][l] = x;
+        else
+            tb->NF[tab - 32][v][l] = x;
+    }
+    // NL: lane-specific shift 16*(31-l)
+    for (int e = t; e < 8 * 16 * 32; e += blockDim.x) {
+        const int q = e / 512, v = (e >> 5) & 15, l = e & 31;
+        tb->NL[q][v][l] = multmodp(x8n(x2n, 16u * (31 - l)), (uint32_t)v << (4 * q));
+    }
+    if (t < kX2n) cs->x2n[t] = x2n[t];
+    if (t < kWarps) cs->warp_shift[t] = x8n(x2n, (uint64_t)(kWarps - 1 - t) * kWarpBytes);
+    if (t == 0) cs->x8n_stride = x8n(x2n, (uint64_t)kThreads * 16);
 }
 
 __global__ void k_setup_geometry(uint32_t *tile_shift, uint32_t *chunk_shift, uint32_t *ff, const CrcConsts *cs,
                                  uint64_t cb, uint32_t n, uint32_t tpc) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i < tpc) {
-        uint64_t end = (uint64_t)(i + 1) * kTile;
+    if (i < tpc * kWarps) {  // sub-tile (t, w) = warp w's 8 KiB of tile t
+        uint64_t end = (uint64_t)(i / kWarps) * kTile + (uint64_t)(i % kWarps + 1) * kWarpBytes;
         if (end > cb) end = cb;
         tile_shift[i] = x8n(cs->x2n, cb - end);
     }
@@ -128,31 +149,41 @@ struct RowCursor {
     }
 };
 
-__device__ __forceinline__ uint4 load_bytes(uint64_t addr, uint32_t k) {
-    uint32_t w[4] = {0, 0, 0, 0};
-    const uint8_t *s = reinterpret_cast<const uint8_t *>(addr);
+// Slow path for a word whose source is misaligned or shorter than 16 bytes (tensor tail).
+// Never reads past the row: k bytes only.  No local-memory arrays (64-bit halves).
+__device__ __noinline__ uint4 load_bytes(uint64_t addr, uint32_t k) {
+    uint64_t lo = 0, hi = 0;
     if (k == 16 && (addr & 3) == 0) {
         const uint32_t *s4 = reinterpret_cast<const uint32_t *>(addr);
-#pragma unroll
-        for (int i = 0; i < 4; ++i) w[i] = __ldg(s4 + i);
-    } else {
-        for (uint32_t i = 0; i < k; ++i) w[i >> 2] |= (uint32_t)__ldg(s + i) << (8 * (i & 3));
+        return make_uint4(__ldg(s4), __ldg(s4 + 1), __ldg(s4 + 2), __ldg(s4 + 3));
     }
-    return make_uint4(w[0], w[1], w[2], w[3]);
+    const uint8_t *s = reinterpret_cast<const uint8_t *>(addr);
+    for (uint32_t i = 0; i < k; ++i) {
+        const uint64_t b = __ldg(s + i);
+        if (i < 8)
+            lo |= b << (8 * i);
+        else
+            hi |= b << (8 * (i - 8));
+    }
+    return make_uint4((uint32_t)lo, (uint32_t)(lo >> 32), (uint32_t)hi, (uint32_t)(hi >> 32));
 }
 
-__device__ __forceinline__ void store_bytes(uint64_t addr, uint32_t k, uint4 v) {
-    const uint32_t w[4] = {v.x, v.y, v.z, v.w};
+__device__ __noinline__ void store_bytes(uint64_t addr, uint32_t k, uint4 v) {
     if (k == 16 && (addr & 15) == 0) {
         *reinterpret_cast<uint4 *>(addr) = v;
-    } else if (k == 16 && (addr & 3) == 0) {
-        uint32_t *d = reinterpret_cast<uint32_t *>(addr);
-#pragma unroll
-        for (int i = 0; i < 4; ++i) d[i] = w[i];
-    } else {
-        uint8_t *d = reinterpret_cast<uint8_t *>(addr);
-        for (uint32_t i = 0; i < k; ++i) d[i] = (uint8_t)(w[i >> 2] >> (8 * (i & 3)));
+        return;
     }
+    if (k == 16 && (addr & 3) == 0) {
+        uint32_t *d = reinterpret_cast<uint32_t *>(addr);
+        d[0] = v.x;
+        d[1] = v.y;
+        d[2] = v.z;
+        d[3] = v.w;
+        return;
+    }
+    const uint64_t lo = ((uint64_t)v.y << 32) | v.x, hi = ((uint64_t)v.w << 32) | v.z;
+    uint8_t *d = reinterpret_cast<uint8_t *>(addr);
+    for (uint32_t i = 0; i < k; ++i) d[i] = (uint8_t)(i < 8 ? lo >> (8 * i) : hi >> (8 * (i - 8)));
 }
 
 // gather the 16-byte image word at chunk position p
@@ -171,59 +202,84 @@ __device__ __forceinline__ void scatter_word(RowCursor &rc, uint32_t p, uint4 v)
 }
 
 // ------------------------------------------------------------------------- K1 / K2
+__device__ __forceinline__ void cp_async16(uint32_t sdst, const void *gsrc) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sdst), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+__device__ __forceinline__ uint4 lds128(uint32_t a) {
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a) : "memory");
+    return v;
+}
+__device__ __forceinline__ void sts128(uint32_t a, uint4 v) {
+    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+
+// Puts the image word at chunk position p into this lane's staging slot `slot`:
+// cp.async for a full, 16-B aligned source word (the common case), else a register path
+// (tensor tail, misaligned view, pad) that stores the word into the slot itself.
+__device__ __forceinline__ void stage_word(RowCursor &rc, uint32_t p, uint32_t slot) {
+    uint64_t addr = 0;
+    const uint32_t k = rc.at(p, addr);
+    if (k == 16 && (addr & 15) == 0)
+        cp_async16(slot, reinterpret_cast<const void *>(addr));
+    else
+        sts128(slot, k ? load_bytes(addr, k) : make_uint4(0, 0, 0, 0));
+}
+
 template <bool kPack>
-__device__ __forceinline__ uint32_t tile_fast(const SnapParams &P, const CrcTables &tb, char *chunk,
-                                              const uint32_t *warp_shift, uint32_t *warp_crc, int rb, int re,
-                                              uint32_t tile0) {
+__device__ __forceinline__ void tile_fast(const SnapParams &P, const CrcTables &tb, char *chunk,
+                                          const SegRow *rows, int nrows, uint32_t tile0, uint32_t stage_base,
+                                          uint32_t *crc_out) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint32_t wbase = tile0 + warp * kWarpBytes;
+    const uint32_t lane4 = lane * 4;
+    const uint32_t wbase = tile0 + warp * kWarpBytes + lane * 16;
+    const uint32_t slot0 = stage_base + (warp * kStages * kRound) + lane * 16;  // this lane's ring
+    const char *nf = reinterpret_cast<const char *>(&tb.NF[0][0][0]);
     RowCursor rc;
-    rc.init(P.rows, rb, re, wbase + lane * 16);
-    uint4 w[kRounds];
-    if (kPack) {
+    rc.init(rows, 0, nrows, wbase);
+    auto issue = [&](int r) {
+        const uint32_t slot = slot0 + (r % kStages) * kRound;
+        if (kPack)
+            stage_word(rc, wbase + r * kRound, slot);
+        else
+            cp_async16(slot, chunk + wbase + r * kRound);
+    };
 #pragma unroll
-        for (int r = 0; r < kRounds; ++r) w[r] = gather_word(rc, wbase + r * kRound + lane * 16);
-#pragma unroll
-        for (int r = 0; r < kRounds; ++r) st_stream(chunk + wbase + r * kRound + lane * 16, w[r]);
-    } else {
-#pragma unroll
-        for (int r = 0; r < kRounds; ++r) w[r] = ld_stream(chunk + wbase + r * kRound + lane * 16);
+    for (int r = 0; r < kStages; ++r) {
+        issue(r);
+        cp_async_commit();
     }
     uint32_t s = 0;
 #pragma unroll
     for (int r = 0; r < kRounds; ++r) {
-        s = shift4(tb.G, s);
-        s = update16(tb.T, s, w[r]);
+        cp_async_wait<kStages - 1>();  // round r's group has landed (one group per round)
+        const uint4 w = lds128(slot0 + (r % kStages) * kRound);
+        if (kPack) st_stream(chunk + wbase + r * kRound, w);
+        s = nib8(nf, lane4, s) ^ raw16(tb, lane4, w);
+        if (!kPack) scatter_word(rc, wbase + r * kRound, w);
+        if (r + kStages < kRounds) issue(r + kStages);
+        cp_async_commit();
     }
-    if (!kPack) {
+    // lane -> end of this warp's 8 KiB (NL tables), XOR over the warp: the sub-tile's raw CRC
+    s = nib8(reinterpret_cast<const char *>(&tb.NL[0][0][0]), lane4, s);
 #pragma unroll
-        for (int r = 0; r < kRounds; ++r) scatter_word(rc, wbase + r * kRound + lane * 16, w[r]);
-    }
-    // lanes -> warp: level k joins groups of 2^k lanes; the right group spans 16*2^k bytes
-#pragma unroll
-    for (int k = 0; k < 5; ++k) {
-        const uint32_t o = __shfl_up_sync(0xFFFFFFFFu, s, 1 << k);
-        if ((lane & ((2 << k) - 1)) == (2 << k) - 1) s = shift4(tb.L[k], o) ^ s;
-    }
-    if (lane == 31) warp_crc[warp] = multmodp(warp_shift[warp], s);
-    __syncthreads();
-    uint32_t t = 0;
-    if (threadIdx.x == 0) {
-#pragma unroll
-        for (int i = 0; i < kWarps; ++i) t ^= warp_crc[i];
-    }
-    return t;  // valid in thread 0
+    for (int o = 16; o > 0; o >>= 1) s ^= __shfl_xor_sync(0xFFFFFFFFu, s, o);
+    if (lane == 0) crc_out[warp] = s;
 }
 
-// Ragged tile (tile_len < kTile, a multiple of 16): block-strided words, generic shifts.
+// Ragged tile (tile_len < kTile, a multiple of 16; only the last tile of a chunk): block-
+// strided words, generic shifts; the whole tile's CRC goes to the last sub-tile slot.
 template <bool kPack>
-__device__ __noinline__ uint32_t tile_generic(const SnapParams &P, const CrcTables &tb, char *chunk,
-                                              uint32_t *warp_crc, int rb, int re, uint32_t tile0,
-                                              uint32_t tile_len) {
+__device__ __noinline__ void tile_generic(const SnapParams &P, const CrcTables &tb, char *chunk,
+                                          const SegRow *rows, int nrows, uint32_t tile0, uint32_t tile_len,
+                                          uint32_t *crc_out, uint32_t *red) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t tile_end = tile0 + tile_len;
     RowCursor rc;
-    rc.init(P.rows, rb, re, tile0 + threadIdx.x * 16);
+    rc.init(rows, 0, nrows, tile0 + threadIdx.x * 16);
     uint32_t s = 0, e = 0;
     bool any = false;
     for (uint32_t p = tile0 + threadIdx.x * 16; p < tile_end; p += kThreads * 16) {
@@ -235,53 +291,104 @@ __device__ __noinline__ uint32_t tile_generic(const SnapParams &P, const CrcTabl
             w = ld_stream(chunk + p);
             scatter_word(rc, p, w);
         }
-        if (any) s = multmodp(P.consts->x8n_stride_gap, s);
-        s = update16(tb.T, s, w);
+        if (any) s = multmodp(P.consts->x8n_stride, s);
+        s ^= raw16(tb, lane * 4, w);
         e = p + 16;
         any = true;
     }
     uint32_t c = any ? multmodp(x8n(P.consts->x2n, tile_end - e), s) : 0u;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) c ^= __shfl_xor_sync(0xFFFFFFFFu, c, o);
-    if (lane == 0) warp_crc[warp] = c;
+    if (lane == 0) red[warp] = c;
     __syncthreads();
-    uint32_t t = 0;
-    if (threadIdx.x == 0) {
-        for (int i = 0; i < kWarps; ++i) t ^= warp_crc[i];
+    if (threadIdx.x < kWarps) {
+        uint32_t t = 0;
+        if (threadIdx.x == kWarps - 1)
+            for (int i = 0; i < kWarps; ++i) t ^= red[i];
+        crc_out[threadIdx.x] = t;  // slot kWarps-1 is relative to tile_end == chunk end
     }
-    return t;
+}
+
+// The 96 KiB of tables arrive in shared memory by one TMA bulk copy (cp.async.bulk, completion
+// on an mbarrier) while the first tile's rows are being staged.
+__device__ __forceinline__ void tables_async_load(void *smem, const void *gmem, uint32_t bytes, uint64_t *bar) {
+    const uint32_t sbar = (uint32_t)__cvta_generic_to_shared(bar);
+    const uint32_t sdst = (uint32_t)__cvta_generic_to_shared(smem);
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(sbar));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sbar), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(sdst),
+                 "l"(gmem), "r"(bytes), "r"(sbar)
+                 : "memory");
+}
+
+__device__ __forceinline__ void tables_wait(uint64_t *bar) {
+    const uint32_t sbar = (uint32_t)__cvta_generic_to_shared(bar);
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], 0;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(sbar)
+        : "memory");
+}
+
+__device__ __forceinline__ uint2 item_rows(const SnapParams &P, uint32_t item, uint32_t n_items) {
+    if (item >= n_items) return make_uint2(0, 0);
+    const uint32_t jl = item / P.tpc, t = item - jl * P.tpc;
+    return P.tile_rows[(uint64_t)(P.first + jl) * P.tpc + t];
+}
+
+// cp.async (LDGSTS) of a tile's segment rows into one of two shared buffers; one commit group
+__device__ __forceinline__ void stage_rows(const SnapParams &P, uint2 tr, SegRow *dst) {
+    const uint32_t k = tr.y <= (uint32_t)kMaxTileRows ? tr.y : 0u;
+    for (uint32_t i = threadIdx.x; i < k; i += kThreads) {
+        const uint32_t sd = (uint32_t)__cvta_generic_to_shared(dst + i);
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sd), "l"(P.rows + tr.x + i) : "memory");
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
 }
 
 template <bool kPack>
-__global__ void __launch_bounds__(kThreads) k_snapshot(const SnapParams P) {
-    extern __shared__ __align__(16) uint8_t smem[];
+__global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
+    // dynamic shared memory: [CrcTables 96 KiB][per-warp cp.async staging rings 96 KiB]
+    extern __shared__ __align__(128) uint8_t smem[];
     CrcTables &tb = *reinterpret_cast<CrcTables *>(smem);
-    __shared__ uint32_t warp_crc[kWarps];
-    __shared__ uint32_t warp_shift[kWarps];
-    {
-        const uint4 *g = reinterpret_cast<const uint4 *>(P.tables);
-        uint4 *d = reinterpret_cast<uint4 *>(smem);
-        for (int i = threadIdx.x; i < (int)(sizeof(CrcTables) / 16); i += kThreads) d[i] = g[i];
-        if (threadIdx.x < kWarps) warp_shift[threadIdx.x] = P.consts->warp_shift[threadIdx.x];
-    }
-    __syncthreads();
+    const uint32_t stage_base = (uint32_t)__cvta_generic_to_shared(smem + sizeof(CrcTables));
+    __shared__ __align__(16) SegRow srows[2][kMaxTileRows];
+    __shared__ uint32_t red[kWarps];
+    __shared__ __align__(8) uint64_t tbar;
     const uint32_t n_items = P.count * P.tpc;
-    for (uint32_t item = blockIdx.x; item < n_items; item += gridDim.x) {
+    const uint32_t G = gridDim.x;
+    uint32_t item = blockIdx.x;
+    uint2 tr = item_rows(P, item, n_items);
+    if (threadIdx.x == 0) tables_async_load(smem, P.tables, sizeof(CrcTables), &tbar);
+    stage_rows(P, tr, srows[0]);
+    uint2 trn = item_rows(P, item + G, n_items);
+    __syncthreads();  // mbarrier initialised before anyone waits on it
+    tables_wait(&tbar);
+    for (int buf = 0; item < n_items; item += G, buf ^= 1) {
+        cp_async_wait<0>();  // this tile's rows (the only group in flight here)
+        __syncthreads();
+        stage_rows(P, trn, srows[buf ^ 1]);  // the next tile's rows, in flight during this one
+        const uint2 trnn = item_rows(P, item + 2 * G, n_items);
+        const SegRow *rows = tr.y <= (uint32_t)kMaxTileRows ? srows[buf] : P.rows + tr.x;
         const uint32_t jl = item / P.tpc, t = item - jl * P.tpc;
         const uint32_t j = P.first + jl;
         char *chunk = P.ring_base + ((P.ring_head + j) % P.ring_slots) * P.chunk_bytes;
         const uint32_t tile0 = t * kTile;
         const uint64_t rem = P.chunk_bytes - tile0;
-        const uint32_t tile_len = rem < kTile ? (uint32_t)rem : kTile;
-        const int rb = P.row_begin[j], re = P.row_begin[j + 1];
-        uint32_t crc;
-        if (tile_len == kTile)
-            crc = tile_fast<kPack>(P, tb, chunk, warp_shift, warp_crc, rb, re, tile0);
+        uint32_t *crc_out = P.tile_crc + ((uint64_t)j * P.tpc + t) * kWarps;
+        if (rem >= kTile)
+            tile_fast<kPack>(P, tb, chunk, rows, (int)tr.y, tile0, stage_base, crc_out);
         else
-            crc = tile_generic<kPack>(P, tb, chunk, warp_crc, rb, re, tile0, tile_len);
-        if (threadIdx.x == 0) P.tile_crc[(uint64_t)j * P.tpc + t] = crc;
-        __syncthreads();  // warp_crc reuse
+            tile_generic<kPack>(P, tb, chunk, rows, (int)tr.y, tile0, (uint32_t)rem, crc_out, red);
+        __syncthreads();  // srows[buf] and red[] are reused
+        tr = trn;
+        trn = trnn;
     }
+    cp_async_wait<0>();
 }
 
 // tiles -> chunk CRC (+ verify) -> slice digest.  One CTA per chunk.
@@ -289,8 +396,9 @@ __global__ void __launch_bounds__(256) k_finalize(const FinalizeParams F) {
     __shared__ uint32_t red[8];
     const uint32_t j = blockIdx.x;
     uint32_t v = 0;
-    for (uint32_t t = threadIdx.x; t < F.tpc; t += blockDim.x)
-        v ^= multmodp(F.tile_shift[t], F.tile_crc[(uint64_t)j * F.tpc + t]);
+    const uint32_t nsub = F.tpc * kWarps;
+    for (uint32_t t = threadIdx.x; t < nsub; t += blockDim.x)
+        v ^= multmodp(F.tile_shift[t], F.tile_crc[(uint64_t)j * nsub + t]);
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v ^= __shfl_xor_sync(0xFFFFFFFFu, v, o);
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;
@@ -361,10 +469,10 @@ cudaError_t setup_geometry(DevGeometry *g, uint64_t chunk_bytes, uint32_t n, cud
     g->chunk_bytes = chunk_bytes;
     g->n = n;
     g->tpc = (uint32_t)((chunk_bytes + kTile - 1) / kTile);
-    if ((e = cudaMalloc(&g->tile_shift, sizeof(uint32_t) * g->tpc)) != cudaSuccess) return e;
+    if ((e = cudaMalloc(&g->tile_shift, sizeof(uint32_t) * g->tpc * kWarps)) != cudaSuccess) return e;
     if ((e = cudaMalloc(&g->chunk_shift, sizeof(uint32_t) * (n ? n : 1))) != cudaSuccess) return e;
     if ((e = cudaMalloc(&g->ff, sizeof(uint32_t) * 2)) != cudaSuccess) return e;
-    const uint32_t m = g->tpc > n ? g->tpc : (n ? n : 1);
+    const uint32_t m = g->tpc * kWarps > n ? g->tpc * kWarps : (n ? n : 1);
     k_setup_geometry<<<(m + 255) / 256, 256, 0, s>>>(g->tile_shift, g->chunk_shift, g->ff, cs, chunk_bytes, n, g->tpc);
     return cudaGetLastError();
 }
@@ -381,9 +489,9 @@ static int resident_ctas(int device) {
     if (device < 0 || device >= 64) return 1;
     if (!cached[device]) {
         int per_sm = 0, sms = 0;
-        cudaFuncSetAttribute(k_snapshot<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sizeof(CrcTables));
-        cudaFuncSetAttribute(k_snapshot<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sizeof(CrcTables));
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snapshot<true>, kThreads, sizeof(CrcTables));
+        cudaFuncSetAttribute(k_snapshot<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sizeof(CrcTables) + kStageBytes);
+        cudaFuncSetAttribute(k_snapshot<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sizeof(CrcTables) + kStageBytes);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snapshot<true>, kThreads, sizeof(CrcTables) + kStageBytes);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
         cached[device] = (per_sm > 0 ? per_sm : 1) * (sms > 0 ? sms : 1);
     }
@@ -399,13 +507,13 @@ int snapshot_grid(int device, uint32_t n_items, uint32_t cap) {
 
 cudaError_t launch_pack(const SnapParams &p, int grid, cudaStream_t s) {
     if (p.count == 0) return cudaSuccess;
-    k_snapshot<true><<<grid, kThreads, sizeof(CrcTables), s>>>(p);
+    k_snapshot<true><<<grid, kThreads, sizeof(CrcTables) + kStageBytes, s>>>(p);
     return cudaGetLastError();
 }
 
 cudaError_t launch_unpack(const SnapParams &p, int grid, cudaStream_t s) {
     if (p.count == 0) return cudaSuccess;
-    k_snapshot<false><<<grid, kThreads, sizeof(CrcTables), s>>>(p);
+    k_snapshot<false><<<grid, kThreads, sizeof(CrcTables) + kStageBytes, s>>>(p);
     return cudaGetLastError();
 }
 

@@ -22,7 +22,7 @@ struct DevGeometry {
     uint64_t chunk_bytes = 0;
     uint32_t n = 0;              // chunks in this rank's slice
     uint32_t tpc = 0;            // tiles per chunk = ceil(chunk_bytes / kTile)
-    uint32_t *tile_shift = nullptr;   // [tpc]  x8n(CB - end of tile t)
+    uint32_t *tile_shift = nullptr;   // [tpc*kWarps] x8n(CB - end of sub-tile (t, w)) (a sub-tile = one warp's 8 KiB)
     uint32_t *chunk_shift = nullptr;  // [n]    x8n((n-1-j) * CB)
     uint32_t *ff = nullptr;           // [2]    shift(~0, CB), shift(~0, n*CB)
 };
@@ -33,18 +33,19 @@ struct DevGeometry {
 struct SnapParams {
     const SegRow *rows;
     const uint32_t *row_begin;   // [n+1] rows of slice chunk j: [row_begin[j], row_begin[j+1])
+    const uint2 *tile_rows;      // [n*tpc] rows overlapping tile (j, t): x = first row index, y = count
     uint64_t chunk_bytes;
     uint32_t first, count, tpc;
     char *ring_base;
     uint64_t ring_head, ring_slots;
-    uint32_t *tile_crc;          // [n * tpc] raw tile CRCs
+    uint32_t *tile_crc;          // [n * tpc * kWarps] raw sub-tile CRCs (relative to each sub-tile's end)
     const CrcTables *tables;
     const CrcConsts *consts;
 };
 
 struct FinalizeParams {
     const uint32_t *tile_crc;
-    uint32_t n, tpc;
+    uint32_t n, tpc;             // sub-tiles per chunk = tpc * kWarps
     const uint32_t *tile_shift, *chunk_shift, *ff;
     uint32_t *crc_out;           // [n] standard CRC32C per chunk
     const uint32_t *expect;      // restore: [n] expected CRCs (nullptr when packing)

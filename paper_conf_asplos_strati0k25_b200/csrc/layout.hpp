@@ -8,6 +8,7 @@
 // of the slice, the pieces of tensors that land in it; K1 gathers them, K2 scatters them.
 #pragma once
 #include <cstdint>
+#include <algorithm>
 #include <vector>
 
 #include "../../include/pccheck.h"
@@ -21,7 +22,26 @@ struct HostLayout {
     uint64_t first = 0, n = 0;      // chunk range the rows describe
     std::vector<SegRow> rows;       // sorted by (chunk, dst_off)
     std::vector<uint32_t> row_begin;  // [n+1]
+    std::vector<uint32_t> tile_rows;  // [2*n*tpc] (first row, count) of the rows overlapping each K1 tile
 };
+
+// Rows overlapping each tile [t*tile, (t+1)*tile) of each chunk (K1 stages them in shared memory).
+inline void build_tile_rows(HostLayout *L, uint64_t cb, uint32_t tile) {
+    const uint64_t tpc = (cb + tile - 1) / tile;
+    L->tile_rows.assign(2 * L->n * tpc, 0);
+    for (uint64_t j = 0; j < L->n; ++j) {
+        uint32_t r = L->row_begin[j];
+        const uint32_t re = L->row_begin[j + 1];
+        for (uint64_t t = 0; t < tpc; ++t) {
+            const uint64_t t0 = t * tile, t1 = std::min<uint64_t>(t0 + tile, cb);
+            while (r < re && (uint64_t)L->rows[r].dst_off + L->rows[r].len <= t0) ++r;
+            uint32_t e = r;
+            while (e < re && L->rows[e].dst_off < t1) ++e;
+            L->tile_rows[2 * (j * tpc + t)] = r;
+            L->tile_rows[2 * (j * tpc + t) + 1] = e - r;
+        }
+    }
+}
 
 inline uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 

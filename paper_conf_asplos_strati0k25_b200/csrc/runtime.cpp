@@ -53,6 +53,20 @@ int cuda_error(cudaError_t e, const char *what) {
 
 using Clock = std::chrono::steady_clock;
 
+// PCC_TRACE=1: one stderr line per pipeline event (debugging hangs on the GPU box)
+static bool trace_on() {
+    static int on = -1;
+    if (on < 0) on = std::getenv("PCC_TRACE") ? 1 : 0;
+    return on;
+}
+#define PCC_TRACE(...)                        \
+    do {                                      \
+        if (trace_on()) {                     \
+            std::fprintf(stderr, "[pcc] " __VA_ARGS__); \
+            std::fputc('\n', stderr);         \
+        }                                     \
+    } while (0)
+
 struct Launch {
     uint32_t first, count;
     cudaEvent_t ev;
@@ -68,8 +82,9 @@ struct Ckpt {
     std::vector<Launch> launches;
     uint32_t launched = 0;  // chunks launched (guarded by mu)
     bool launch_failed = false;
+    bool final_recorded = false;  // ev_final recorded (guarded by mu): finish must not sync it before
     std::atomic<uint32_t> remaining{0};
-    cudaEvent_t ev_train = nullptr, ev_begin = nullptr, ev_packed = nullptr, ev_final = nullptr;
+    cudaEvent_t ev_train = nullptr, ev_begin = nullptr, ev_packed = nullptr, ev_fin_k = nullptr, ev_final = nullptr;
     double t_call = 0, t_packed = 0, t_landed = 0, t_persisted = 0, t_committed = 0;
     float pack_ms = 0, fin_ms = 0;
     uint32_t digest = 0;
@@ -141,6 +156,7 @@ struct pcc_ctx {
     uint64_t first = 0, n = 0;
     SegRow *rows_dev = nullptr;
     uint32_t *row_begin_dev = nullptr;
+    uint2 *tile_rows_dev = nullptr;
     DevGeometry geom;
     SlotGeom sgeom{};
     uint32_t lcrc = 0;
@@ -274,10 +290,17 @@ void fail_ckpt(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck, int err) {
 
 // Listing 1 lines 16-34 for a checkpoint whose chunks are all durable.
 void finish_ckpt(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
+    PCC_TRACE("finish: ckpt %llu", (unsigned long long)ck->t.counter);
+    {
+        // the chunks may all have landed before the training thread recorded ev_final (the
+        // finalize kernel + CRC table copy): syncing an unrecorded event returns at once
+        std::unique_lock<std::mutex> lk(ck->mu);
+        ck->cv.wait(lk, [&] { return ck->final_recorded; });
+    }
     cudaError_t e = cudaEventSynchronize(ck->ev_final);
     if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "finalize"));
     cudaEventElapsedTime(&ck->pack_ms, ck->ev_begin, ck->ev_packed);
-    cudaEventElapsedTime(&ck->fin_ms, ck->ev_packed, ck->ev_final);
+    cudaEventElapsedTime(&ck->fin_ms, ck->ev_packed, ck->ev_fin_k);  // the finalize kernel alone
     const uint32_t *h = c->crc_host[ck->t.slot];
     ck->crc.assign(h, h + c->n);
     ck->digest = h[c->n];
@@ -296,6 +319,7 @@ void finish_ckpt(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
     set_state(c, ck.get(), PCC_ST_PERSISTED);
     int st = PCC_ST_FAILED;
     int rc = c->engine->complete(ck->t, ck->crc.data(), ck->digest, &st);
+    PCC_TRACE("finish: ckpt %llu committed state %d rc %d", (unsigned long long)ck->t.counter, st, rc);
     if (rc) fail_ckpt(c, ck, rc);
     if (c->cfg.world == 1 || st == PCC_ST_FAILED) {
         ck->t_committed = c->now_us();
@@ -309,7 +333,9 @@ void persist_loop(pcc_ctx *c) {
     PersistTask task;
     while (c->tasks.pop(&task)) {
         Ckpt *ck = task.ck.get();
+        PCC_TRACE("persist: ckpt %llu chunk %u wait", (unsigned long long)ck->t.counter, task.j);
         cudaError_t e = cudaEventSynchronize(task.ev);
+        PCC_TRACE("persist: ckpt %llu chunk %u landed (%s)", (unsigned long long)ck->t.counter, task.j, cudaGetErrorString(e));
         if (e != cudaSuccess) fail_ckpt(c, task.ck, cuda_error(e, "chunk copy"));
         if (task.pooled_ev) put_event(c, task.ev);
         if (!c->zerocopy()) ring_release(c, ck->ring_start + task.j);
@@ -325,6 +351,7 @@ void persist_loop(pcc_ctx *c) {
             std::lock_guard<std::mutex> lk(ck->mu);
             ck->t_landed = std::max(ck->t_landed, t);
         }
+        PCC_TRACE("persist: ckpt %llu chunk %u done", (unsigned long long)ck->t.counter, task.j);
         if (ck->remaining.fetch_sub(1) == 1) finish_ckpt(c, task.ck);
     }
 }
@@ -333,11 +360,14 @@ void orchestrate_loop(pcc_ctx *c) {
     cudaSetDevice(c->device);
     std::shared_ptr<Ckpt> ck;
     while (c->jobs.pop(&ck)) {
+        PCC_TRACE("orch: ckpt %llu iter %llu slot %u", (unsigned long long)ck->t.counter,
+                  (unsigned long long)ck->t.iter, ck->t.slot);
         if (c->fd >= 0) {
             int rc = c->engine->filling(ck->t);  // R18: before any data byte of this slot changes
             if (rc) fail_ckpt(c, ck, rc);
         }
         size_t li = 0;
+        uint32_t issued = 0;
         for (uint32_t j = 0; j < c->n; ++j) {
             Launch L;
             {
@@ -355,6 +385,7 @@ void orchestrate_loop(pcc_ctx *c) {
                 if (j == L.first) cudaStreamWaitEvent(c->copy_stream, L.ev, 0);
                 task.dest = c->mapfile() ? c->map + c->slot_data_off(ck->t.slot) + (uint64_t)j * c->cb()
                                          : staging_acquire(c);
+                PCC_TRACE("orch: ckpt %llu chunk %u -> %p", (unsigned long long)ck->t.counter, j, (void *)task.dest);
                 const char *src = c->ring + ((ck->ring_start + j) % c->ring_slots) * c->cb();
                 cudaError_t e = cudaMemcpyAsync(task.dest, src, c->cb(), cudaMemcpyDeviceToHost, c->copy_stream);
                 if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "D2H"));
@@ -363,16 +394,21 @@ void orchestrate_loop(pcc_ctx *c) {
                 cudaEventRecord(task.ev, c->copy_stream);
             }
             c->tasks.push(task);
+            ++issued;
         }
-        if (c->n == 0) finish_ckpt(c, ck);
+        // chunks never issued (K1 launch failed) count as done so the checkpoint still terminates
+        const uint32_t unissued = (uint32_t)c->n - issued;
+        if (c->n == 0 || (unissued && ck->remaining.fetch_sub(unissued) == unissued)) finish_ckpt(c, ck);
     }
 }
 
 int free_registration(pcc_ctx *c) {
     cudaFree(c->rows_dev);
     cudaFree(c->row_begin_dev);
+    cudaFree(c->tile_rows_dev);
     c->rows_dev = nullptr;
     c->row_begin_dev = nullptr;
+    c->tile_rows_dev = nullptr;
     free_geometry(&c->geom);
     for (auto p : c->tile_crc_dev) cudaFree(p);
     for (auto p : c->crc_dev) cudaFree(p);
@@ -402,6 +438,7 @@ void destroy_ckpt_events(pcc_ctx *c, Ckpt *ck) {
     cudaEventDestroy(ck->ev_train);
     cudaEventDestroy(ck->ev_begin);
     cudaEventDestroy(ck->ev_packed);
+    cudaEventDestroy(ck->ev_fin_k);
     cudaEventDestroy(ck->ev_final);
     for (auto &L : ck->launches) put_event(c, L.ev);
     ck->launches.clear();
@@ -543,6 +580,7 @@ int pcc_register(pcc_ctx *c, const pcc_tensor *t, uint32_t nt) {
     slice_of(full.C, c->cfg.rank, c->cfg.world, &c->first, &c->n);
     rc = build_layout(t, nt, c->cfg.align, c->cb(), c->first, (int64_t)c->n, &c->layout);
     if (rc) return set_error(PCC_EINVAL, "layout slice");
+    build_tile_rows(&c->layout, c->cb(), kTile);
     std::vector<uint64_t> nb(nt);
     std::vector<uint32_t> dt(nt);
     for (uint32_t i = 0; i < nt; ++i) {
@@ -560,12 +598,20 @@ int pcc_register(pcc_ctx *c, const pcc_tensor *t, uint32_t nt) {
     if (!c->layout.rows.empty())
         cudaMemcpy(c->rows_dev, c->layout.rows.data(), c->layout.rows.size() * sizeof(SegRow), cudaMemcpyHostToDevice);
     cudaMemcpy(c->row_begin_dev, c->layout.row_begin.data(), (c->n + 1) * sizeof(uint32_t), cudaMemcpyHostToDevice);
+    {
+        const size_t tb = std::max<size_t>(c->layout.tile_rows.size(), 2) * sizeof(uint32_t);
+        if ((e = cudaMalloc(&c->tile_rows_dev, tb)) != cudaSuccess) return cuda_error(e, "tile rows");
+        if (!c->layout.tile_rows.empty())
+            cudaMemcpy(c->tile_rows_dev, c->layout.tile_rows.data(), c->layout.tile_rows.size() * sizeof(uint32_t),
+                       cudaMemcpyHostToDevice);
+    }
     if ((e = setup_geometry(&c->geom, c->cb(), (uint32_t)c->n, c->pack_stream)) != cudaSuccess)
         return cuda_error(e, "geometry");
     const uint64_t nn = c->n ? c->n : 1;
     for (uint32_t s = 0; s < c->n_slots; ++s) {
         uint32_t *a = nullptr, *b = nullptr, *d = nullptr, *h = nullptr;
-        if ((e = cudaMalloc(&a, nn * c->geom.tpc * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "tile crc");
+        if ((e = cudaMalloc(&a, nn * c->geom.tpc * kWarps * sizeof(uint32_t))) != cudaSuccess)
+            return cuda_error(e, "tile crc");
         if ((e = cudaMalloc(&b, (nn + 1) * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "crc");
         if ((e = cudaMalloc(&d, 4 * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "scratch");
         if ((e = cudaMallocHost(&h, (nn + 1) * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "crc host");
@@ -666,6 +712,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
     cudaEventCreateWithFlags(&ck->ev_train, cudaEventDisableTiming);
     cudaEventCreate(&ck->ev_begin);
     cudaEventCreate(&ck->ev_packed);
+    cudaEventCreate(&ck->ev_fin_k);
     cudaEventCreateWithFlags(&ck->ev_final, cudaEventDisableTiming);
     cudaEventRecord(ck->ev_train, ts);
     cudaStreamWaitEvent(c->pack_stream, ck->ev_train, 0);
@@ -680,6 +727,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
     SnapParams P{};
     P.rows = c->rows_dev;
     P.row_begin = c->row_begin_dev;
+    P.tile_rows = c->tile_rows_dev;
     P.chunk_bytes = c->cb();
     P.tpc = c->geom.tpc;
     P.tile_crc = c->tile_crc_dev[s];
@@ -697,9 +745,12 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
         c->launches += c->n ? 1 : 0;
         cudaEvent_t ev = get_event(c);
         cudaEventRecord(ev, c->pack_stream);
-        std::lock_guard<std::mutex> lk(ck->mu);
-        ck->launches.push_back({0, (uint32_t)c->n, ev});
-        ck->launched = (uint32_t)c->n;
+        {
+            std::lock_guard<std::mutex> lk(ck->mu);
+            ck->launches.push_back({0, (uint32_t)c->n, ev});
+            ck->launched = (uint32_t)c->n;
+        }
+        ck->cv.notify_all();  // the orchestrator may already be waiting for this launch
     } else {  // Variant B: HBM ring, windowed by ring space
         {
             std::lock_guard<std::mutex> lk(c->ring_mu);
@@ -749,18 +800,21 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
     F.crc_out = c->crc_dev[s];
     F.scratch = c->scratch_dev[s];
     if (e == cudaSuccess) e = launch_finalize(F, c->pack_stream);
+    cudaEventRecord(ck->ev_fin_k, c->pack_stream);
     if (c->n) c->launches += 1;
     cudaMemcpyAsync(c->crc_dev[s] + c->n, c->scratch_dev[s] + 3, 4, cudaMemcpyDeviceToDevice, c->pack_stream);
     cudaMemcpyAsync(c->crc_host[s], c->crc_dev[s], (c->n + 1) * sizeof(uint32_t), cudaMemcpyDeviceToHost,
                     c->pack_stream);
     cudaEventRecord(ck->ev_final, c->pack_stream);
-    if (e != cudaSuccess) {
-        int rc = cuda_error(e, "K1 launch");
-        fail_ckpt(c, ck, rc);
+    {
         std::lock_guard<std::mutex> lk(ck->mu);
-        ck->launch_failed = true;
-        ck->cv.notify_all();
+        ck->final_recorded = true;
+        if (e != cudaSuccess) {
+            fail_ckpt(c, ck, cuda_error(e, "K1 launch"));
+            ck->launch_failed = true;
+        }
     }
+    ck->cv.notify_all();
     *out = ck->t.counter;
     return PCC_OK;
 }
@@ -1026,7 +1080,7 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     };
     if (!v.ok || !v.layout_ok) return done(set_error(PCC_ELAYOUT, "slot header"));
     if ((e = cudaMalloc(&expect, n * 4)) || (e = cudaMalloc(&bad, n * 4)) || (e = cudaMalloc(&crc, n * 4)) ||
-        (e = cudaMalloc(&tile, n * c->geom.tpc * 4)) || (e = cudaMalloc(&scr, 16)))
+        (e = cudaMalloc(&tile, n * c->geom.tpc * kWarps * 4)) || (e = cudaMalloc(&scr, 16)))
         return done(cuda_error(e, "restore buffers"));
     cudaMemcpy(expect, v.crc, n * 4, cudaMemcpyHostToDevice);
     cudaMemset(scr, 0, 16);
@@ -1042,6 +1096,7 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     SnapParams P{};
     P.rows = c->rows_dev;
     P.row_begin = c->row_begin_dev;
+    P.tile_rows = c->tile_rows_dev;
     P.chunk_bytes = cb;
     P.tpc = c->geom.tpc;
     P.ring_base = ring;

@@ -44,3 +44,10 @@ def load_golden_crc():
             name, hx, crc = line.split()
             out.append((name, b"" if hx == "-" else bytes.fromhex(hx), int(crc, 16)))
     return out
+
+
+def pytest_collection_modifyitems(config, items):
+    # a hung GPU test must fail, not eat the whole gpurun budget
+    for it in items:
+        if it.get_closest_marker("gpu") and not it.get_closest_marker("timeout"):
+            it.add_marker(pytest.mark.timeout(240))
