@@ -319,6 +319,16 @@ def main():
         dist.all_reduce(t2, op=dist.ReduceOp.MAX)
     e2e_value = state_bytes * args.steps / (float(t2.item()) * 1e-3) / 1e9
 
+    # restore (L287 + K2 verify): the newest checkpoint back into the registered tensors
+    restore = None
+    if args.mode != "nullsink" and world == 1:
+        barrier()
+        t0r = time.perf_counter()
+        rit, rbad = ck.restore()
+        torch.cuda.synchronize()
+        rdt = time.perf_counter() - t0r
+        restore = {"iter": rit, "ms": rdt * 1e3, "gbs": state_bytes / rdt / 1e9, "bad_chunks": len(rbad),
+                   "path": "file mapping -> H2D into the HBM ring -> K2 verify+scatter"}
     peak_link = d2h_peak_gbs(torch)
     ck.close()
     if path and os.path.exists(path):
@@ -362,6 +372,7 @@ def main():
                               "frac": link_achieved / peak_link,
                               "peak_source": "pinned 1 GiB cudaMemcpy D2H, measured in this run"},
             "finalize_ms": fin_ms,
+            "restore": restore,
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": state_bytes,
                     "d2h_bytes_per_step": slice_bytes + 4 * (geo["count"] + 1)},
