@@ -49,6 +49,16 @@ PCC_API int pcc_host_geometry(pcc_host *h, uint32_t *first, uint32_t *n, uint32_
 PCC_API uint64_t pcc_host_data_offset(pcc_host *h, uint32_t slot);
 /* held (committed, not freed) iters: writes up to cap (iter, slot) pairs, returns count */
 PCC_API uint32_t pcc_host_held(pcc_host *h, uint64_t *iters, uint32_t *slots, uint32_t cap);
+
+/* The restore agreement of pcc_restore (R8, R10) over this engine's rank file,
+ * with the collectives and the slice verification supplied by the caller: `reduce` performs an
+ * in-place allreduce of one int64 across ranks (is_max: MAX else MIN; identity for W = 1),
+ * `verify` checks this rank's slice of `iter` in `slot` (0 = intact).  COLLECTIVE: every rank
+ * calls it with the same want_iter / flags.  Returns 0 and *restored_iter, or -PCC_E*. */
+typedef int (*pcc_reduce_fn)(void *ctx, int64_t *value, int is_max);
+typedef int (*pcc_verify_fn)(void *ctx, uint64_t iter, uint32_t slot);
+PCC_API int pcc_host_restore_plan(pcc_host *h, uint64_t want_iter, uint32_t flags, pcc_reduce_fn reduce,
+                                  pcc_verify_fn verify, void *ctx, uint64_t *restored_iter);
 PCC_API int pcc_host_close(pcc_host *h);
 
 #ifdef __cplusplus

@@ -96,8 +96,11 @@ _SIGS = {
     "pcc_host_geometry": (C.c_int, [_P, _u32p, _u32p, _u32p]),
     "pcc_host_data_offset": (C.c_uint64, [_P, C.c_uint32]),
     "pcc_host_held": (C.c_uint32, [_P, _u64p, _u32p, C.c_uint32]),
+    "pcc_host_restore_plan": (C.c_int, [_P, C.c_uint64, C.c_uint32, _P, _P, _P, _u64p]),
     "pcc_host_close": (C.c_int, [_P]),
 }
+REDUCE_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.POINTER(C.c_int64), C.c_int)
+VERIFY_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_uint64, C.c_uint32)
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_lib, _name)
     _f.restype = _res
@@ -356,6 +359,24 @@ class HostEngine:
         sl = (C.c_uint32 * 64)()
         k = _lib.pcc_host_held(self._h, it, sl, 64)
         return {it[i]: sl[i] for i in range(min(k, 64))}
+
+    def restore_plan(self, reduce, verify, want_iter=None, fallback=False):
+        """reduce(value:int, is_max:bool) -> int (an allreduce across ranks); verify(iter, slot) -> bool."""
+        def _r(ctx, v, is_max):
+            v[0] = int(reduce(int(v[0]), bool(is_max)))
+            return 0
+
+        def _v(ctx, it, slot):
+            return 0 if verify(int(it), int(slot)) else 1
+
+        rf, vf = REDUCE_FN(_r), VERIFY_FN(_v)
+        out = C.c_uint64()
+        rc = _lib.pcc_host_restore_plan(self._h, LATEST if want_iter is None else want_iter,
+                                        FALLBACK if fallback else 0, C.cast(rf, C.c_void_p), C.cast(vf, C.c_void_p),
+                                        None, C.byref(out))
+        if rc != 0:
+            raise PCCError(rc, "pcc_host_restore_plan")
+        return out.value
 
     def close(self):
         if self._h:

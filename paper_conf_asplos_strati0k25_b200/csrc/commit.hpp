@@ -106,4 +106,30 @@ class CommitEngine {
     ~CommitEngine();
 };
 
+// ------------------------------------------------------------------ restore agreement
+// What a rank file holds (FORMAT.md): the valid pointer record with the largest seq and the
+// iters of COMPLETE, CRC-valid headers (split by whether they match the registration).
+struct SlotScan {
+    std::map<uint64_t, uint32_t> complete;    // iter -> slot
+    std::map<uint64_t, uint32_t> bad_layout;  // iter -> slot, header valid but another registration
+    PtrRecord best;
+};
+int scan_rank_file(int fd, const SlotGeom &g, uint32_t n_slots, SlotScan *S);
+
+// The restore protocol of L287 (§4.2) with verification, for W ranks:
+// every rank runs the same control flow, steered only by reduced values, so the collectives
+// match.  W = 1 passes an identity reducer.
+//   g = MAX_r(global_iter of the rank's best record)   (or want_iter)
+//   loop: all = MIN_r(g is held COMPLETE here); if all: verify own slice (K2), err = MAX_r(err);
+//         no error -> fanout (W > 1) -> done;  else (PCC_FALLBACK) g = MIN_r(max{h held < g})
+struct RestoreOps {
+    std::function<int(int64_t *v, bool is_max)> reduce;                           // in place, 1 value
+    std::function<int(uint64_t iter, uint32_t slot, std::vector<uint32_t> *bad)> verify;  // own slice
+    std::function<int(uint64_t iter, uint32_t slot)> fanout;                     // W > 1 (may be empty)
+};
+// Returns PCC_OK with *restored set, or the first candidate's error; *bad_first receives
+// this rank's failing chunk indices of that first rejected candidate.
+int restore_agree(const SlotScan &S, uint64_t want_iter, uint32_t flags, const RestoreOps &ops, uint64_t *restored,
+                  std::vector<uint32_t> *bad_first);
+
 }  // namespace pcc

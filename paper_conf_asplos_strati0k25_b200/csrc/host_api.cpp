@@ -136,6 +136,23 @@ uint32_t pcc_host_held(pcc_host *h, uint64_t *iters, uint32_t *slots, uint32_t c
     return k;
 }
 
+int pcc_host_restore_plan(pcc_host *h, uint64_t want_iter, uint32_t flags, pcc_reduce_fn reduce, pcc_verify_fn verify,
+                          void *ctx, uint64_t *restored_iter) {
+    if (!h || !reduce || !verify || h->fd < 0) return set_error(PCC_EINVAL, "args");
+    SlotScan S;
+    int rc = scan_rank_file(h->fd, h->engine.geom(), h->n_slots, &S);
+    if (rc) return rc;
+    RestoreOps ops;
+    ops.reduce = [&](int64_t *v, bool is_max) { return reduce(ctx, v, is_max ? 1 : 0); };
+    ops.verify = [&](uint64_t it, uint32_t slot, std::vector<uint32_t> *) {
+        return verify(ctx, it, slot) == 0 ? PCC_OK : set_error(PCC_ECORRUPT, "verify callback");
+    };
+    uint64_t it = 0;
+    rc = restore_agree(S, want_iter, flags, ops, &it, nullptr);
+    if (rc == PCC_OK && restored_iter) *restored_iter = it;
+    return rc;
+}
+
 int pcc_host_close(pcc_host *h) {
     if (!h) return PCC_OK;
     int fd = h->fd;

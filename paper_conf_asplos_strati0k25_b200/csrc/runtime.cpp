@@ -1023,36 +1023,6 @@ int pread_full(int fd, char *p, uint64_t n, uint64_t off) {
     return PCC_OK;
 }
 
-struct SlotScan {
-    std::map<uint64_t, uint32_t> complete;  // iter -> slot (COMPLETE, header CRC ok, layout ok)
-    std::map<uint64_t, uint32_t> bad_layout;
-    PtrRecord best;
-};
-
-int scan_file(pcc_ctx *c, SlotScan *S) {
-    uint8_t *buf = static_cast<uint8_t *>(std::aligned_alloc(kPage, header_bytes(c->n)));
-    if (!buf) return set_error(PCC_ENOMEM, "scan buffer");
-    for (int k = 0; k < 2; ++k) {
-        if (::pread(c->fd, buf, kPage, k * kPage) != (ssize_t)kPage) continue;
-        PtrRecord r = decode_ptr(buf);
-        if (r.valid && r.rank == (uint32_t)c->cfg.rank && r.world == (uint32_t)c->cfg.world &&
-            (!S->best.valid || r.seq > S->best.seq))
-            S->best = r;
-    }
-    const uint64_t H = header_bytes(c->n);
-    for (uint32_t s = 0; s < c->n_slots; ++s) {
-        if (::pread(c->fd, buf, H, slot_offset(s, c->n, c->cb())) != (ssize_t)H) continue;
-        HeaderView v = decode_header(buf, c->sgeom, s);
-        if (!v.ok) continue;
-        if (v.layout_ok)
-            S->complete[v.iter] = s;
-        else
-            S->bad_layout[v.iter] = s;
-    }
-    std::free(buf);
-    return PCC_OK;
-}
-
 // K2 over this rank's slice of the checkpoint in `slot`: H2D into the HBM ring, verify every
 // chunk's CRC32C against the header table while scattering into the registered tensors.
 int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
@@ -1084,6 +1054,7 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
         return done(cuda_error(e, "restore buffers"));
     cudaMemcpy(expect, v.crc, n * 4, cudaMemcpyHostToDevice);
     cudaMemset(scr, 0, 16);
+    PCC_TRACE("restore: slot %u buffers ready t=%.0f us", slot, c->now_us());
     // ring for restore: zero-copy mode has none; allocate one batch worth
     char *ring = c->ring;
     uint64_t R = c->ring_slots;
@@ -1131,6 +1102,7 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
         cudaEventRecord(ev, c->pack_stream);
         cudaStreamWaitEvent(c->copy_stream, ev, 0);  // next batch's H2D after this K2 read the ring
     }
+    PCC_TRACE("restore: copies + K2 issued t=%.0f us", c->now_us());
     FinalizeParams F{};
     F.tile_crc = tile;
     F.n = (uint32_t)n;
@@ -1152,6 +1124,7 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
         if ((e = cudaStreamSynchronize(c->pack_stream))) rc = cuda_error(e, "restore sync");
     }
     cudaStreamSynchronize(c->copy_stream);
+    PCC_TRACE("restore: verified t=%.0f us", c->now_us());
     put_event(c, ev);
     if (own_ring) cudaFree(ring);
     if (rc) return done(rc);
@@ -1162,10 +1135,130 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     return done(PCC_OK);
 }
 
-int restore_dp(pcc_ctx *c, SlotScan *S, uint64_t want_iter, uint32_t flags, uint64_t *restored_iter,
-               uint32_t *bad_chunks, uint32_t bad_cap, uint32_t *n_bad) {
-    (void)S; (void)want_iter; (void)flags; (void)restored_iter; (void)bad_chunks; (void)bad_cap; (void)n_bad;
-    return set_error(PCC_ESTATE, "world > 1 restore not built yet");
+// C3 of SURVEY §2.3: after every rank verified (and scattered) its own slice of iter g, the
+// verified packed chunks cross NVLink with ncclAllGather in groups of G chunks per rank, and
+// each rank K2-verifies + scatters the other ranks' chunks into its registered tensors (the
+// CRC tables travel too, so a transfer fault is caught).  Uneven slices are padded to
+// n_max = ceil(C / W) chunks per rank.
+int dp_fanout(pcc_ctx *c, uint32_t slot) {
+    const uint64_t cb = c->cb(), C = c->layout.C;
+    const uint32_t W = (uint32_t)c->cfg.world, me = (uint32_t)c->cfg.rank;
+    const uint64_t n_max = (C + W - 1) / W;
+    if (C == 0) return PCC_OK;
+    // full-image segment table (every chunk, not just this rank's slice)
+    HostLayout full;
+    if (build_layout(c->tensors.data(), (uint32_t)c->tensors.size(), c->cfg.align, cb, 0, -1, &full))
+        return set_error(PCC_EINVAL, "full layout");
+    build_tile_rows(&full, cb, kTile);
+    SegRow *rows = nullptr;
+    uint32_t *rb = nullptr, *tile = nullptr, *crc_mine = nullptr, *crc_all = nullptr, *crc_out = nullptr, *bad = nullptr,
+             *scr = nullptr;
+    uint2 *trows = nullptr;
+    char *send = nullptr, *recv = nullptr;
+    DevGeometry g2;
+    cudaError_t e = cudaSuccess;
+    int rc = PCC_OK;
+    auto done = [&](int r) {
+        cudaFree(rows); cudaFree(rb); cudaFree(tile); cudaFree(crc_mine); cudaFree(crc_all); cudaFree(crc_out);
+        cudaFree(bad); cudaFree(scr); cudaFree(trows); cudaFree(send); cudaFree(recv);
+        free_geometry(&g2);
+        return r;
+    };
+    // group size: bounded by 4 GiB of receive buffer
+    uint64_t G = std::max<uint64_t>(1, std::min<uint64_t>(n_max, (4ull << 30) / (W * cb)));
+    const uint64_t nsub = (uint64_t)c->geom.tpc * kWarps;
+    if ((e = cudaMalloc(&rows, std::max<size_t>(1, full.rows.size()) * sizeof(SegRow))) ||
+        (e = cudaMalloc(&rb, (C + 1) * 4)) || (e = cudaMalloc(&trows, std::max<size_t>(2, full.tile_rows.size()) * 4)) ||
+        (e = cudaMalloc(&tile, C * nsub * 4)) || (e = cudaMalloc(&crc_mine, n_max * 4)) ||
+        (e = cudaMalloc(&crc_all, W * n_max * 4)) || (e = cudaMalloc(&crc_out, C * 4)) || (e = cudaMalloc(&bad, C * 4)) ||
+        (e = cudaMalloc(&scr, 16 * W)) || (e = cudaMalloc(&send, G * cb)) || (e = cudaMalloc(&recv, W * G * cb)))
+        return done(cuda_error(e, "fanout buffers"));
+    if (!full.rows.empty()) cudaMemcpy(rows, full.rows.data(), full.rows.size() * sizeof(SegRow), cudaMemcpyHostToDevice);
+    cudaMemcpy(rb, full.row_begin.data(), (C + 1) * 4, cudaMemcpyHostToDevice);
+    if (!full.tile_rows.empty()) cudaMemcpy(trows, full.tile_rows.data(), full.tile_rows.size() * 4, cudaMemcpyHostToDevice);
+    if ((e = setup_geometry(&g2, cb, (uint32_t)n_max, c->pack_stream))) return done(cuda_error(e, "fanout geometry"));
+    // this rank's CRC table (from its slot header) -> allgather
+    {
+        const uint64_t H = header_bytes(c->n);
+        uint8_t *hdr = static_cast<uint8_t *>(std::aligned_alloc(kPage, H));
+        rc = pread_full(c->fd, reinterpret_cast<char *>(hdr), H, slot_offset(slot, c->n, cb));
+        std::vector<uint32_t> mine(n_max, 0);
+        if (rc == PCC_OK) std::memcpy(mine.data(), hdr + 96, c->n * 4);
+        std::free(hdr);
+        if (rc) return done(rc);
+        cudaMemcpy(crc_mine, mine.data(), n_max * 4, cudaMemcpyHostToDevice);
+    }
+    if ((rc = c->nccl.allgather(crc_mine, crc_all, n_max * 4, c->pack_stream))) return done(rc);
+    const uint64_t data0 = c->slot_data_off(slot);
+    std::vector<uint64_t> first_q(W), n_q(W);
+    for (uint32_t q = 0; q < W; ++q) slice_of(C, q, W, &first_q[q], &n_q[q]);
+    uint32_t launches = 0;
+    for (uint64_t k0 = 0; k0 < n_max && rc == PCC_OK; k0 += G) {
+        const uint64_t mine_k = n_q[me] > k0 ? std::min<uint64_t>(G, n_q[me] - k0) : 0;
+        for (uint64_t i = 0; i < mine_k && rc == PCC_OK; ++i) {  // own verified chunks -> send buffer
+            const char *src;
+            if (c->mapfile()) {
+                src = c->map + data0 + (k0 + i) * cb;
+            } else {
+                char *st = c->staging + (i % c->staging_slots) * cb;
+                if (i >= c->staging_slots) cudaStreamSynchronize(c->copy_stream);
+                rc = pread_full(c->fd, st, cb, data0 + (k0 + i) * cb);
+                src = st;
+            }
+            if (rc == PCC_OK) cudaMemcpyAsync(send + i * cb, src, cb, cudaMemcpyHostToDevice, c->copy_stream);
+        }
+        cudaStreamSynchronize(c->copy_stream);
+        if (rc) break;
+        if ((rc = c->nccl.allgather(send, recv, G * cb, c->pack_stream))) break;
+        for (uint32_t q = 0; q < W; ++q) {
+            if (q == me) continue;
+            const uint64_t cnt = n_q[q] > k0 ? std::min<uint64_t>(G, n_q[q] - k0) : 0;
+            if (!cnt) continue;
+            const uint64_t j0 = first_q[q] + k0;  // global chunk index
+            SnapParams P{};
+            P.rows = rows;
+            P.row_begin = rb;
+            P.tile_rows = trows;
+            P.chunk_bytes = cb;
+            P.first = (uint32_t)j0;
+            P.count = (uint32_t)cnt;
+            P.tpc = c->geom.tpc;
+            P.ring_base = recv + (uint64_t)q * G * cb;
+            P.ring_slots = 1ull << 40;
+            P.ring_head = P.ring_slots - j0;
+            P.tile_crc = tile;
+            P.tables = c->tables;
+            P.consts = c->consts;
+            if ((e = launch_unpack(P, snapshot_grid(c->device, (uint32_t)(cnt * P.tpc), 0), c->pack_stream))) {
+                rc = cuda_error(e, "fanout K2");
+                break;
+            }
+            FinalizeParams F{};
+            F.tile_crc = tile + j0 * nsub;
+            F.n = (uint32_t)cnt;
+            F.tpc = c->geom.tpc;
+            F.tile_shift = g2.tile_shift;
+            F.chunk_shift = g2.chunk_shift;
+            F.ff = g2.ff;
+            F.crc_out = crc_out + j0;
+            F.expect = crc_all + (uint64_t)q * n_max + k0;
+            F.bad = bad + j0;
+            F.scratch = scr + 4 * q;
+            cudaMemsetAsync(F.scratch, 0, 16, c->pack_stream);
+            if ((e = launch_finalize(F, c->pack_stream))) {
+                rc = cuda_error(e, "fanout finalize");
+                break;
+            }
+            launches += 2;
+        }
+        if ((e = cudaStreamSynchronize(c->pack_stream))) rc = cuda_error(e, "fanout sync");  // recv reused next group
+        std::vector<uint32_t> sc(4 * W);
+        cudaMemcpy(sc.data(), scr, 16 * W, cudaMemcpyDeviceToHost);
+        for (uint32_t q = 0; q < W && rc == PCC_OK; ++q)
+            if (sc[4 * q + 2]) rc = set_error(PCC_ECORRUPT, "chunk corrupted in the NVLink fan-out");
+    }
+    c->launches += launches;
+    return done(rc);
 }
 
 }  // namespace
@@ -1178,41 +1271,27 @@ extern "C" int pcc_restore(pcc_ctx *c, uint64_t want_iter, uint32_t flags, uint6
     if (c->fd < 0) return set_error(PCC_ENOENT, "no file (NULLSINK)");
     pcc_drain(c, -1);
     cudaSetDevice(c->device);
+    PCC_TRACE("restore: start t=%.0f us", c->now_us());
     SlotScan S;
-    int rc = scan_file(c, &S);
+    int rc = scan_rank_file(c->fd, c->sgeom, c->n_slots, &S);
     if (rc) return rc;
-    if (c->cfg.world > 1) return restore_dp(c, &S, want_iter, flags, restored_iter, bad_chunks, bad_cap, n_bad);
-    uint64_t target = want_iter;
-    if (target == PCC_LATEST) {
-        if (!S.best.valid) return set_error(PCC_ENOENT, "no valid pointer record");
-        target = S.best.global_iter;
+    PCC_TRACE("restore: scanned t=%.0f us", c->now_us());
+    RestoreOps ops;
+    if (c->cfg.world == 1) {
+        ops.reduce = [](int64_t *, bool) { return PCC_OK; };
+    } else {
+        ops.reduce = [c](int64_t *v, bool is_max) {
+            return c->nccl.allreduce_i64(v, 1, is_max ? NcclComm::kMax : NcclComm::kMin, c->red_dev, c->red_host,
+                                         c->aux_stream);
+        };
+        ops.fanout = [c](uint64_t, uint32_t slot) { return dp_fanout(c, slot); };
     }
-    int first_rc = 0;
-    bool reported = false;
-    for (;;) {
-        int cand;
-        std::vector<uint32_t> bad;
-        auto it = S.complete.find(target);
-        if (it == S.complete.end()) {
-            cand = S.bad_layout.count(target) ? set_error(PCC_ELAYOUT, "registration differs from checkpoint")
-                                               : set_error(PCC_ENOENT, "iter not held");
-        } else {
-            cand = verify_scatter(c, it->second, &bad);
-        }
-        if (cand == PCC_OK) {
-            if (restored_iter) *restored_iter = target;
-            return PCC_OK;
-        }
-        if (!reported) {
-            reported = true;
-            first_rc = cand;
-            if (n_bad) *n_bad = (uint32_t)bad.size();
-            for (size_t i = 0; i < bad.size() && i < bad_cap && bad_chunks; ++i) bad_chunks[i] = bad[i];
-        }
-        if (!(flags & PCC_FALLBACK)) return first_rc;
-        auto lower = S.complete.lower_bound(target);  // first >= target
-        if (lower == S.complete.begin()) return first_rc;
-        --lower;
-        target = lower->first;
-    }
+    ops.verify = [c](uint64_t, uint32_t slot, std::vector<uint32_t> *bad) { return verify_scatter(c, slot, bad); };
+    uint64_t it = 0;
+    std::vector<uint32_t> bad;
+    rc = restore_agree(S, want_iter, flags, ops, &it, &bad);
+    if (n_bad) *n_bad = (uint32_t)bad.size();
+    for (size_t i = 0; i < bad.size() && i < bad_cap && bad_chunks; ++i) bad_chunks[i] = bad[i];
+    if (rc == PCC_OK && restored_iter) *restored_iter = it;
+    return rc;
 }

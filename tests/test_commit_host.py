@@ -220,3 +220,82 @@ def test_dp_commit_gloo_world2(tmp_path, seed):
     rc, it, bad, outs = oracle.restore(paths, 3, SIZES, [0] * len(SIZES), 256, CB)
     assert rc == 0 and it == g
     assert all(np.array_equal(o, x) for o, x in zip(outs, _state(g)))
+
+
+# ----------------------------------------------- restore agreement under gloo (pcc_restore's W>1 logic)
+def _verify_with_oracle(path, e, slot):
+    """The test's stand-in for K2 on this rank's slice: recompute every chunk CRC32C with the
+    oracle and compare with the slot header's table."""
+    import struct as _s
+    first, n, _ = e.geometry()
+    with open(path, "rb") as f:
+        f.seek(oracle.slot_offset(slot, n, CB))
+        hdr = f.read(oracle.header_bytes(n))
+        f.seek(e.data_offset(slot))
+        data = np.frombuffer(f.read(n * CB), dtype=np.uint8)
+    if data.nbytes < n * CB:
+        return False
+    table = list(_s.unpack_from(f"<{n}I", hdr, 96)) if n else []
+    return [int(x) for x in oracle.chunk_crcs(data, CB)] == table
+
+
+def _agree_worker(rank, world, tmpdir, scenario, q):
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        path = os.path.join(tmpdir, f"r{rank}.pcc")
+        e = _engine(path, 2, rank, world)
+        for it in (10, 20, 30):
+            counter, slot = e.begin(it)
+            e.filling(counter)
+            if not (scenario == "rank1_missing_30" and rank == 1 and it == 30):  # else: 30 never durable here
+                crcs, dig = _write_data(e, path, slot, _state(it), rank, world)
+                e.complete(counter, crcs, dig)
+            L = torch.tensor([e.local_latest()])
+            dist.all_reduce(L, op=dist.ReduceOp.MIN)
+            e.apply_global(int(L.item()))
+        if scenario == "corrupt_rank1_latest" and rank == 1:
+            held = e.held()
+            g = e.global_iter()
+            with open(path, "r+b") as f:
+                f.seek(e.data_offset(held[g]) + 123)
+                b = f.read(1)
+                f.seek(e.data_offset(held[g]) + 123)
+                f.write(bytes([b[0] ^ 0x80]))
+
+        def reduce(v, is_max):
+            t = torch.tensor([v], dtype=torch.int64)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX if is_max else dist.ReduceOp.MIN)
+            return int(t.item())
+
+        try:
+            got = e.restore_plan(reduce, lambda it, slot: _verify_with_oracle(path, e, slot), fallback=True)
+        except pcc.PCCError as ex:
+            got = -ex.code
+        e.close()
+        q.put((rank, got))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("scenario", ["clean", "rank1_missing_30", "corrupt_rank1_latest"])
+def test_restore_agreement_gloo_world2(tmp_path, scenario):
+    import torch.multiprocessing as mp
+    os.environ["MASTER_PORT"] = str(31500 + (os.getpid() + len(scenario)) % 2000)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_agree_worker, args=(r, 2, str(tmp_path), scenario, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(120)
+        assert p.exitcode == 0
+    res = dict(q.get() for _ in range(2))
+    assert res[0] == res[1], res  # every rank restores the same iter
+    paths = [str(tmp_path / f"r{r}.pcc") for r in range(2)]
+    rc, it, bad, outs = oracle.restore(paths, 3, SIZES, [0] * len(SIZES), 256, CB, fallback=True)
+    assert rc == 0 and res[0] == it  # ... the one the oracle picks from the same files
+    expect = {"clean": 30, "rank1_missing_30": 20, "corrupt_rank1_latest": 20}[scenario]
+    assert it == expect
