@@ -200,6 +200,8 @@ def main():
     ap.add_argument("--no-slowdown", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--mode", default="mapfile", choices=["mapfile", "zerocopy", "nullsink", "pwrite"])
+    ap.add_argument("--emulate-world", type=int, default=0,
+                    help="1 GPU plays rank 0 of this world size alone (PCC_NOCOMM): per-GPU share of a DP job")
     args = ap.parse_args()
     rank, world = env_int("RANK", 0), env_int("WORLD_SIZE", 1)
     local = env_int("LOCAL_RANK", 0)
@@ -229,15 +231,22 @@ def main():
     from paper_conf_asplos_strati0k25_b200 import k_layout
     n_est = k_layout([(1 << 20, s.nbytes, s.code) for s in specs], 256, cb)[2]
     slice_est = -(-n_est // world) * cb
+    emu = args.emulate_world if world == 1 and args.emulate_world > 1 else 0
+    if emu:
+        slice_est = -(-n_est // emu) * cb
     flags = {"mapfile": pcc.MAPFILE, "zerocopy": pcc.MAPFILE | pcc.ZEROCOPY, "nullsink": pcc.NULLSINK,
-             "pwrite": pcc.ODIRECT}[args.mode]
+             "pwrite": pcc.ODIRECT}[args.mode] | (pcc.NOCOMM if emu else 0)
     shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
     path = None if args.mode == "nullsink" else os.path.join(shm, f"pcc_bench_{os.getpid()}_r{rank}.pcc")
     ck = pcc.PCCheck(path, chunk_bytes=cb, max_inflight=args.inflight, flags=flags, device=local, rank=rank,
-                     world=world, nccl_unique_id=uid, staging_bytes=8 * cb, ring_bytes=args.ring_slices * slice_est)
+                     world=emu or world, nccl_unique_id=uid, staging_bytes=8 * cb, ring_bytes=args.ring_slices * slice_est)
     ck.register(state)
     geo = ck.geometry()
     slice_bytes = geo["count"] * cb
+    if emu:  # state bytes inside this rank's chunk range (R3: GB/s counts state bytes, not pads)
+        offs, _, _ = pcc.k_layout([(1 << 20, s.nbytes, s.code) for s in specs], 256, cb)
+        lo, hi = geo["first"] * cb, (geo["first"] + geo["count"]) * cb
+        state_bytes = sum(max(0, min(o + s.nbytes, hi) - max(o, lo)) for o, s in zip(offs, specs))
     stream = torch.cuda.current_stream()
 
     def barrier():
@@ -293,17 +302,23 @@ def main():
     value = state_bytes * args.steps / (ms_total * 1e-3) / 1e9  # whole job (every rank packs its 1/W slice)
 
     # ---- e2e: the state comes from pinned host memory every step (H2D inside the timed region)
-    host_state = [torch.empty_like(s, device="cpu").pin_memory() for s in state]
-    for h_, d_ in zip(host_state, state):
-        h_.copy_(d_)
+    # the inputs of this rank's share: every tensor overlapping its chunk range (all of them at W=1)
+    offs_all, _, _ = pcc.k_layout([(1 << 20, s.nbytes, s.code) for s in specs], 256, cb)
+    lo_b, hi_b = geo["first"] * cb, (geo["first"] + geo["count"]) * cb
+    upload = [i for i, (o, s) in enumerate(zip(offs_all, specs)) if o < hi_b and o + s.nbytes > lo_b]
+    h2d_bytes = sum(specs[i].nbytes for i in upload)
+    host_state = {i: torch.empty_like(state[i], device="cpu").pin_memory() for i in upload}
+    for i, h_ in host_state.items():
+        h_.copy_(state[i])
     barrier()
     e2 = torch.cuda.Event(enable_timing=True)
     e3 = torch.cuda.Event(enable_timing=True)
     e2.record(stream)
     hs2 = []
-    for _ in range(args.steps):
-        for h_, d_ in zip(host_state, state):
-            d_.copy_(h_, non_blocking=True)
+    e2e_steps = args.steps if state_bytes < (8 << 30) else min(args.steps, 3)  # bounded for 10-100 GB states
+    for _ in range(e2e_steps):
+        for i, h_ in host_state.items():
+            state[i].copy_(h_, non_blocking=True)
         hs2.append(one_ckpt())
     crc_bytes = 0
     for h in hs2:
@@ -317,7 +332,7 @@ def main():
     t2 = torch.tensor([e2.elapsed_time(e3)], device="cuda")
     if world > 1:
         dist.all_reduce(t2, op=dist.ReduceOp.MAX)
-    e2e_value = state_bytes * args.steps / (float(t2.item()) * 1e-3) / 1e9
+    e2e_value = state_bytes * e2e_steps / (float(t2.item()) * 1e-3) / 1e9
 
     # restore (L287 + K2 verify): the newest checkpoint back into the registered tensors
     restore = None
@@ -335,12 +350,18 @@ def main():
         os.unlink(path)
 
     slowdown = None
-    if rank == 0 and world == 1 and not args.no_slowdown and args.config == "c2":
+    if rank == 0 and world == 1 and not args.no_slowdown and args.config in ("c2", "c4"):
         try:
-            from tools.slowdown import vgg16_slowdown
-            slowdown = vgg16_slowdown(pcc, iters=60, every=10)
+            if args.config == "c2":
+                from tools.slowdown import vgg16_slowdown
+                slowdown = vgg16_slowdown(pcc, iters=60, every=10)
+            else:
+                del state, host_state
+                torch.cuda.empty_cache()
+                from tools.slowdown import bloom_slowdown
+                slowdown = bloom_slowdown(pcc, world=emu or 8, iters=40, every=10)
         except Exception as ex:  # noqa: BLE001
-            slowdown = {"error": repr(ex)[:200]}
+            slowdown = {"error": repr(ex)[:300]}
 
     if rank == 0:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -349,7 +370,7 @@ def main():
         k1_achieved = k1_bytes / (pack_ms * 1e-3) / 1e9
         link_achieved = slice_bytes / (ms_total * 1e-3 / args.steps) / 1e9
         cpu = None
-        if not args.no_cpu_baseline:
+        if not args.no_cpu_baseline and args.config in ("c1", "c2", "c3"):
             cpu = cpu_baseline(specs, state, cb)
         line = {
             "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
@@ -358,7 +379,8 @@ def main():
             "data": "synthetic (seeded bit patterns; shapes of the model's params + optimizer state)",
             "config": {"workload": WORKLOADS.get(args.config, args.config), "config": args.config,
                        "state_bytes": state_bytes, "chunk_bytes": cb, "chunks": geo["n_chunks"],
-                       "inflight": args.inflight, "mode": args.mode, "hbm_ring_slices": args.ring_slices, "parallelism": f"dp{world}",
+                       "inflight": args.inflight, "mode": args.mode, "hbm_ring_slices": args.ring_slices,
+                       "emulated_rank_of_world": emu or None, "parallelism": f"dp{world}",
                        "target": "DRAM file on /dev/shm (tmpfs), mmap + cudaHostRegister" if args.mode != "nullsink"
                        else "null sink", "l2": "inputs larger than L2 (state >> 126 MB)"},
             "per_gpu_gbs": value / world,
@@ -374,7 +396,7 @@ def main():
             "finalize_ms": fin_ms,
             "restore": restore,
             "cpu_baseline": cpu,
-            "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": state_bytes,
+            "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": h2d_bytes,
                     "d2h_bytes_per_step": slice_bytes + 4 * (geo["count"] + 1)},
             "gpu_launches": launches,
             "clocks": clk,

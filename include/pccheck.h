@@ -70,6 +70,10 @@ enum {
     PCC_MAPFILE = 1u << 4,  /* the file's slots are mmap'd + cudaHostRegister'ed: the copy
                                engine (or K1 with ZEROCOPY) writes straight into the file's
                                pages (DRAM-backed file, e.g. tmpfs); persist = fdatasync only */
+    PCC_NOCOMM = 1u << 5,   /* world > 1 without NCCL: this process alone plays rank `rank` of
+                               `world` (packs, persists and commits only its 1/world slice; the
+                               global commit reduces over itself).  For measuring one rank's
+                               share on one GPU; a restore then covers only this slice. */
 };
 
 /* ---- per-checkpoint states (pcc_poll) — SURVEY §8(b) state machine ------------------- */

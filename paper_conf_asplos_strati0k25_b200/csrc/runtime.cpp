@@ -549,7 +549,7 @@ int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
         if (c->fd < 0) return set_errno_error("open checkpoint file", errno);
         c->odirect = flags & O_DIRECT;
     }
-    if (cfg->world > 1) {
+    if (cfg->world > 1 && !(cfg->flags & PCC_NOCOMM)) {
         if (!cfg->nccl_unique_id) return set_error(PCC_EINVAL, "nccl_unique_id required for world > 1");
         int rc = c->nccl.init(cfg->nccl_unique_id, cfg->world, cfg->rank);
         if (rc) return rc;
@@ -879,20 +879,27 @@ int pcc_drain(pcc_ctx *c, int64_t timeout_us) {
     return PCC_OK;
 }
 
+// In-place allreduce of int64 values over the library's NCCL communicator.  PCC_NOCOMM (one
+// process measuring one rank's share alone) reduces over itself.
+static int reduce_i64(pcc_ctx *c, int64_t *v, size_t n, NcclComm::Op op) {
+    if (c->cfg.world == 1 || (c->cfg.flags & PCC_NOCOMM)) return PCC_OK;
+    return c->nccl.allreduce_i64(v, n, op, c->red_dev, c->red_host, c->aux_stream);
+}
+
 // Collective backpressure (SURVEY §7 "hard parts"): a rank without a free slot cannot just
 // block, because only a g-advance frees slots; every rank runs the same rounds of
 // need = MAX(no free slot), g = MIN(L_r) until nobody needs.
 static int dp_backpressure(pcc_ctx *c) {
     for (int round = 0;; ++round) {
         int64_t v[2] = {c->engine->has_free() ? 0 : 1, 0};
-        int rc = c->nccl.allreduce_i64(v, 1, NcclComm::kMax, c->red_dev, c->red_host, c->aux_stream);
+        int rc = reduce_i64(c, v, 1, NcclComm::kMax);
         if (rc) return rc;
         if (v[0] == 0) return PCC_OK;
         // let local persists progress, then advance g
         c->engine->wait_free(2000);
         uint64_t L = c->engine->local_latest();
         int64_t g[1] = {L == UINT64_MAX ? -1 : (int64_t)L};
-        rc = c->nccl.allreduce_i64(g, 1, NcclComm::kMin, c->red_dev, c->red_host, c->aux_stream);
+        rc = reduce_i64(c, g, 1, NcclComm::kMin);
         if (rc) return rc;
         if (g[0] >= 0) c->engine->apply_global((uint64_t)g[0]);
     }
@@ -907,7 +914,7 @@ int pcc_commit(pcc_ctx *c, uint64_t *committed_iter) {
     }
     uint64_t L = c->engine->local_latest();
     int64_t g[1] = {L == UINT64_MAX ? -1 : (int64_t)L};
-    int rc = c->nccl.allreduce_i64(g, 1, NcclComm::kMin, c->red_dev, c->red_host, c->aux_stream);
+    int rc = reduce_i64(c, g, 1, NcclComm::kMin);
     if (rc) return rc;
     if (g[0] >= 0) rc = c->engine->apply_global((uint64_t)g[0]);
     if (committed_iter) *committed_iter = c->engine->global_iter();
@@ -1280,11 +1287,8 @@ extern "C" int pcc_restore(pcc_ctx *c, uint64_t want_iter, uint32_t flags, uint6
     if (c->cfg.world == 1) {
         ops.reduce = [](int64_t *, bool) { return PCC_OK; };
     } else {
-        ops.reduce = [c](int64_t *v, bool is_max) {
-            return c->nccl.allreduce_i64(v, 1, is_max ? NcclComm::kMax : NcclComm::kMin, c->red_dev, c->red_host,
-                                         c->aux_stream);
-        };
-        ops.fanout = [c](uint64_t, uint32_t slot) { return dp_fanout(c, slot); };
+        ops.reduce = [c](int64_t *v, bool is_max) { return reduce_i64(c, v, 1, is_max ? NcclComm::kMax : NcclComm::kMin); };
+        if (!(c->cfg.flags & PCC_NOCOMM)) ops.fanout = [c](uint64_t, uint32_t slot) { return dp_fanout(c, slot); };
     }
     ops.verify = [c](uint64_t, uint32_t slot, std::vector<uint32_t> *bad) { return verify_scatter(c, slot, bad); };
     uint64_t it = 0;

@@ -91,3 +91,104 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
             "slowdown_pct": (c / b - 1.0) * 100.0,
             "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
             "state_bytes": sum(t.numel() * t.element_size() for t in state)}
+
+
+def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1, path=None):
+    """BLOOM-7b1 (BASELINE configs[3]) on ONE B200 as a proxy for one rank of a world-`world`
+    data-parallel job: the per-GPU compute of DP at micro-batch 1 (forward + backward of the
+    full model on one 2048-token sequence, then a mixed-precision Adam step), checkpointing
+    only this rank's 1/world slice (PCC_NOCOMM) every `every` iterations.  What it cannot
+    show: the gradient allreduce of real DP and W ranks contending for host DRAM.
+
+    State per parameter (R11, R12): bf16 param, fp32 master, fp32 exp_avg, fp32 exp_avg_sq,
+    0-d fp32 step — 1825 tensors, 98.97 GB.  Random init, random token ids."""
+    import torch
+    from transformers import BloomConfig, BloomForCausalLM
+
+    torch.manual_seed(0)
+    cfg = BloomConfig(vocab_size=250880, hidden_size=4096, n_layer=30, n_head=32)
+    with torch.device("cuda"):
+        model = BloomForCausalLM(cfg).to(torch.bfloat16)
+    params = [p for p in model.parameters()]
+    master = [p.detach().float() for p in params]
+    exp_avg = [torch.zeros_like(m) for m in master]
+    exp_avg_sq = [torch.zeros_like(m) for m in master]
+    steps = [torch.zeros((), dtype=torch.float32, device="cuda") for _ in params]
+    state = []
+    for p, m, a, b, st in zip(params, master, exp_avg, exp_avg_sq, steps):
+        state += [p.data, m, a, b, st]
+    ids = torch.randint(0, cfg.vocab_size, (1, seq), device="cuda")
+    stream = torch.cuda.current_stream()
+    lr, b1, b2, eps = 1e-5, 0.9, 0.95, 1e-8
+
+    def fwd_bwd():
+        for p in params:
+            p.grad = None
+        model(input_ids=ids, labels=ids).loss.backward()
+
+    @torch.no_grad()
+    def adam_step():  # mixed-precision Adam (no bias correction), one parameter at a time: no fp32 grad copy
+        for p, m, a, b, st in zip(params, master, exp_avg, exp_avg_sq, steps):
+            g = p.grad.float()
+            st.add_(1.0)
+            a.lerp_(g, 1 - b1)
+            b.mul_(b2).addcmul_(g, g, value=1 - b2)
+            m.addcdiv_(a, b.sqrt().add_(eps), value=-lr)
+            p.copy_(m)
+
+    shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
+    path = path or os.path.join(shm, f"pcc_bloom_{os.getpid()}.pcc")
+    ck = pcc.PCCheck(path, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.MAPFILE | pcc.NOCOMM, rank=0, world=world)
+    ck.register(state)
+    geo = ck.geometry()
+
+    def loop(n, checkpoint, it0):
+        handles = []
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        per = []
+        e0.record(stream)
+        last = e0
+        for i in range(1, n + 1):
+            fwd_bwd()
+            if checkpoint:
+                ck.guard(stream)  # U-gate (L139): the update must not race K1
+            adam_step()
+            if checkpoint and i % every == 0:
+                handles.append(ck.checkpoint(it0 + i, stream))
+                ck.commit()
+            ev = torch.cuda.Event(enable_timing=True)
+            ev.record(stream)
+            per.append((last, ev))
+            last = ev
+        e1.record(stream)
+        e1.synchronize()
+        for h in handles:
+            ck.wait(h)
+        return e0.elapsed_time(e1), sorted(a.elapsed_time(b) for a, b in per)
+
+    for _ in range(warmup):
+        fwd_bwd()
+        adam_step()
+    base_t, ck_t, its_b, its_c = [], [], [], []
+    it0 = 1000
+    for r in range(runs):
+        t, its = loop(iters, False, 0)
+        base_t.append(t)
+        its_b += its
+        t, its = loop(iters, True, it0)
+        it0 += 1000
+        ck_t.append(t)
+        its_c += its
+    ck.drain()
+    ck.close()
+    if os.path.exists(path):
+        os.unlink(path)
+    b, c = statistics.mean(base_t), statistics.mean(ck_t)
+    pct = lambda v, q: sorted(v)[min(len(v) - 1, int(q * len(v)))]  # noqa: E731
+    return {"model": f"bloom-7b1 bf16 + fp32 master Adam, micro-batch 1 x {seq} tokens, random init; "
+                     f"1 GPU playing rank 0 of world {world} (checkpoints its 1/{world} slice)",
+            "every": every, "iters": iters, "runs": runs, "slice_chunks": geo["count"],
+            "slice_bytes": geo["count"] * (64 << 20),
+            "iter_ms_no_ckpt": b / iters, "iter_ms_ckpt": c / iters, "slowdown_pct": (c / b - 1.0) * 100.0,
+            "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
+            "state_bytes": sum(t.numel() * t.element_size() for t in state)}
