@@ -125,6 +125,24 @@ def pack(srcs, align=256, chunk_bytes=4 << 20, first_chunk=0, count=None):
     return out
 
 
+def pack_chunks_sparse(all_nbytes, srcs_by_index, align, chunk_bytes, first_chunk, count):
+    """O2 for chunks [first_chunk, first_chunk+count) of a large registration when only the
+    tensors overlapping those chunks are at hand: the layout (O1) comes from ALL sizes, the
+    byte copy from the given tensors (every other tensor must not overlap the range)."""
+    off, end, c = layout(all_nbytes, align, chunk_bytes)
+    lo, hi = first_chunk * chunk_bytes, (first_chunk + count) * chunk_bytes
+    idx = sorted(srcs_by_index)
+    for i in range(len(all_nbytes)):
+        if int(off[i]) < hi and int(off[i]) + int(all_nbytes[i]) > lo and all_nbytes[i] > 0:
+            assert i in srcs_by_index, f"tensor {i} overlaps the range but was not given"
+    arrs, ptrs = _bufs([srcs_by_index[i] for i in idx])
+    nb, nbp = _u64([all_nbytes[i] for i in idx])
+    offa, offp = _u64([off[i] for i in idx])
+    out = np.empty(count * chunk_bytes, dtype=np.uint8)
+    lib().orc_pack(len(idx), ptrs, nbp, offp, chunk_bytes, first_chunk, count, out.ctypes.data)
+    return out
+
+
 def chunk_crcs(img, chunk_bytes):
     """O3 per chunk: crc[c] = CRC32C(image[c*CB:(c+1)*CB])."""
     img = np.ascontiguousarray(img).view(np.uint8)

@@ -329,3 +329,18 @@ def test_restore_dp_global_iter_and_presence(tmp_path):
     rc, it, bad, outs = oracle.restore(paths, N_SLOTS, SIZES, [1] * len(SIZES), 256, CB, fallback=True)
     assert rc == 0 and it == 10
     assert all(o.tobytes() == s.tobytes() for o, s in zip(outs, s10))
+
+
+def test_pack_chunks_sparse_equals_full_pack():
+    """The sampled-chunk helper used at full sizes is the same O2 image, chunk for chunk."""
+    rng = np.random.default_rng(11)
+    sizes = [int(x) for x in rng.integers(0, 9000, 40)]
+    srcs = [rng.integers(0, 256, n, dtype=np.uint8) for n in sizes]
+    cb = 4096
+    full = oracle.pack(srcs, 256, cb)
+    off, end, c = oracle.layout(sizes, 256, cb)
+    for j in range(c):
+        need = {i: srcs[i] for i in range(len(sizes))
+                if sizes[i] and int(off[i]) < (j + 1) * cb and int(off[i]) + sizes[i] > j * cb}
+        part = oracle.pack_chunks_sparse(sizes, need, 256, cb, j, 1)
+        assert part.tobytes() == full[j * cb:(j + 1) * cb].tobytes()
