@@ -58,36 +58,37 @@ __host__ __device__ inline uint32_t x8n(const uint32_t *x2n, uint64_t n) {
 
 // ---------------------------------------------------------------- kernel geometry
 // One CTA of 32 warps per SM (all warps share one 96 KiB copy of the tables), tile = 256 KiB
-// of one chunk, warp region = 8 KiB = 16 rounds of 512 B.  In round r lane l owns the
-// 16-byte word at warp_base + r*512 + 16*l, so every warp access is 512 contiguous bytes.
-// Loads go global -> shared with cp.async into a per-warp ring of kStages rounds (each lane
-// only ever reads back its own 16-byte slot, so no barrier is needed), keeping
-// 32 warps x 6 x 512 B = 96 KiB per SM in flight without spending registers.
-// Per round a lane's register becomes  s <- shift(s, 512) ^ raw16(w);  after the last
-// round its contribution is shifted to the warp-region end (shift by 16*(31-l)) and
-// XOR-reduced over the warp, giving the sub-tile CRC; the finalize kernel folds sub-tiles,
-// chunks and the slice digest.
+// of one chunk, warp region = 8 KiB = 8 rounds of 1 KiB.  In round r lane l owns the 32 bytes
+// at warp_base + r*1024 + 32*l: one 256-bit load and one 256-bit store per lane, so every warp
+// access is 1 KiB contiguous.  Loads run kAhead rounds ahead in registers.  Per round:
+//     x = shift(s, 992);  s = raw16(w0 ^ x);  s = raw16(w1 ^ s)
+// (feeding a 16-byte word into register r equals raw16 of the word with its first 4 bytes
+// XOR r).  After the last round a lane's register is shifted to its warp-region end
+// (shift by 32*(31-l)) and XOR-reduced over the warp: one raw CRC per 8 KiB sub-tile; the
+// finalize kernel folds sub-tiles, chunks and the slice digest.
 //
 // Lookups are NIBBLE tables replicated once per lane: entry (table t, nibble v) of lane l
 // sits at word (t*16 + v)*32 + l, i.e. always in bank l.  Every shared load of the CRC is
-// therefore conflict-free (1 wavefront), at 2 lookups per byte.  (Byte-indexed slicing-by-16
-// tables cost 1.25 lookups per byte but random indices collide in banks ~2.9-way on average;
-// ncu showed the L1/shared pipe at 81% with that design, K1 at 0.45 of HBM.)
+// therefore conflict-free (1 wavefront), at 36 lookups per 16 bytes.  (Byte-indexed
+// slicing-by-16 tables cost 20 lookups per 16 B, but random indices collide in banks ~2.9-way
+// on average; ncu showed the L1/shared pipe at 81% with that design, K1 at 0.45 of HBM.)
 constexpr int kWarps = 32;
 constexpr int kThreads = kWarps * 32;
-constexpr int kRounds = 16;                        // rounds per warp per tile
-constexpr int kStages = 6;                         // cp.async ring depth per warp (rounds in flight)
-constexpr uint32_t kRound = 512;                   // bytes per warp per round
-constexpr uint32_t kWarpBytes = kRounds * kRound;  // 8 KiB per warp
-constexpr uint32_t kTile = kWarps * kWarpBytes;    // 256 KiB per CTA tile
-constexpr uint32_t kStageBytes = kWarps * kStages * kRound;  // 96 KiB of shared staging per CTA
-constexpr int kMaxTileRows = 512;                  // segment rows staged per tile (more -> read from global)
+constexpr int kWpl = 2;                              // 16-byte words per lane per round
+constexpr uint32_t kLaneSpan = 16 * kWpl;            // 32 B
+constexpr uint32_t kRound = 32 * kLaneSpan;          // 1 KiB per warp per round
+constexpr uint32_t kWarpBytes = 8192;                // 8 KiB per warp per tile
+constexpr int kRounds = kWarpBytes / kRound;         // 8
+constexpr int kAhead = 2;                            // rounds loaded ahead of the CRC
+constexpr uint32_t kGap = kRound - kLaneSpan;        // zero bytes between a lane's spans
+constexpr uint32_t kTile = kWarps * kWarpBytes;      // 256 KiB per CTA tile
+constexpr int kMaxTileRows = 512;                    // segment rows staged per tile (more -> read from global)
 
 // Shared-memory table block (96 KiB), per-lane replicated nibble tables.
 struct CrcTables {
     uint32_t NT[32][16][32];  // NT[q][v][l] = raw16(16-byte word whose nibble q is v, others 0)
-    uint32_t NF[8][16][32];   // NF[q][v][l] = shift(v << 4q, 512): one round
-    uint32_t NL[8][16][32];   // NL[q][v][l] = shift(v << 4q, 16*(31-l)): lane -> warp-region end
+    uint32_t NF[8][16][32];   // NF[q][v][l] = shift(v << 4q, kGap): the zeros before a lane's next span
+    uint32_t NL[8][16][32];   // NL[q][v][l] = shift(v << 4q, kLaneSpan*(31-l)): lane -> warp-region end
 };
 static_assert(sizeof(CrcTables) == 96 * 1024, "table block size");
 
@@ -139,6 +140,7 @@ __device__ __forceinline__ uint32_t nib8(const char *tab, uint32_t lane4, uint32
 }
 
 // raw16(w): CRC register of the 16 bytes w fed into a zero register (32 nibble lookups).
+// raw16(w with w.x ^= r) = the register r after absorbing w.
 __device__ __forceinline__ uint32_t raw16(const CrcTables &tb, uint32_t lane4, uint4 w) {
     const char *t = reinterpret_cast<const char *>(&tb.NT[0][0][0]);
     return nib8(t, lane4, w.x) ^ nib8(t + 8 * 2048, lane4, w.y) ^ nib8(t + 16 * 2048, lane4, w.z) ^

@@ -51,8 +51,8 @@ __global__ void k_build_tables(CrcTables *tb, CrcConsts *cs) {
         const int q = e >> 4, v = e & 15;
         vals[q][v] = raw_byte_at(T0, (q & 1) ? (v << 4) : v, q >> 1);
     }
-    // NF: shift by one round
-    const uint32_t xr = x8n(x2n, kRound);
+    // NF: shift by the gap between a lane's spans
+    const uint32_t xr = x8n(x2n, kGap);
     if (t < 8 * 16) {
         const int q = t >> 4, v = t & 15;
         vals[32 + q][v] = multmodp(xr, (uint32_t)v << (4 * q));
@@ -69,7 +69,7 @@ __global__ void k_build_tables(CrcTables *tb, CrcConsts *cs) {
     // NL: lane-specific shift 16*(31-l)
     for (int e = t; e < 8 * 16 * 32; e += blockDim.x) {
         const int q = e / 512, v = (e >> 5) & 15, l = e & 31;
-        tb->NL[q][v][l] = multmodp(x8n(x2n, 16u * (31 - l)), (uint32_t)v << (4 * q));
+        tb->NL[q][v][l] = multmodp(x8n(x2n, kLaneSpan * (31 - l)), (uint32_t)v << (4 * q));
     }
     if (t < kX2n) cs->x2n[t] = x2n[t];
     if (t < kWarps) cs->warp_shift[t] = x8n(x2n, (uint64_t)(kWarps - 1 - t) * kWarpBytes);
@@ -208,60 +208,78 @@ __device__ __forceinline__ void cp_async16(uint32_t sdst, const void *gsrc) {
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
-__device__ __forceinline__ uint4 lds128(uint32_t a) {
-    uint4 v;
-    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a) : "memory");
+
+struct Span {  // one lane's 32 bytes of a round
+    uint4 a, b;
+};
+
+__device__ __forceinline__ Span ld_span(const void *p) {  // 256-bit streaming load
+    Span v;
+    asm volatile("ld.global.nc.L1::no_allocate.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(v.a.x), "=r"(v.a.y), "=r"(v.a.z), "=r"(v.a.w), "=r"(v.b.x), "=r"(v.b.y), "=r"(v.b.z),
+                   "=r"(v.b.w)
+                 : "l"(p));
     return v;
 }
-__device__ __forceinline__ void sts128(uint32_t a, uint4 v) {
-    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+__device__ __forceinline__ void st_span(void *p, const Span &v) {  // 256-bit streaming store
+    asm volatile("st.global.cs.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(v.a.x), "r"(v.a.y),
+                 "r"(v.a.z), "r"(v.a.w), "r"(v.b.x), "r"(v.b.y), "r"(v.b.z), "r"(v.b.w)
+                 : "memory");
 }
 
-// Puts the image word at chunk position p into this lane's staging slot `slot`:
-// cp.async for a full, 16-B aligned source word (the common case), else a register path
-// (tensor tail, misaligned view, pad) that stores the word into the slot itself.
-__device__ __forceinline__ void stage_word(RowCursor &rc, uint32_t p, uint32_t slot) {
+// The image bytes [p, p+32) (p 32-B aligned in the chunk): one 256-bit load when a single row
+// covers them from a 32-B aligned source, else word by word.
+__device__ __forceinline__ Span gather_span(RowCursor &rc, uint32_t p) {
     uint64_t addr = 0;
     const uint32_t k = rc.at(p, addr);
-    if (k == 16 && (addr & 15) == 0)
-        cp_async16(slot, reinterpret_cast<const void *>(addr));
-    else
-        sts128(slot, k ? load_bytes(addr, k) : make_uint4(0, 0, 0, 0));
+    if (k == 16 && rc.stop - p >= 32 && (addr & 31) == 0) return ld_span(reinterpret_cast<const void *>(addr));
+    Span v;
+    v.a = k == 16 && (addr & 15) == 0 ? ld_stream(reinterpret_cast<const void *>(addr))
+                                       : (k ? load_bytes(addr, k) : make_uint4(0, 0, 0, 0));
+    v.b = gather_word(rc, p + 16);
+    return v;
+}
+
+__device__ __forceinline__ void scatter_span(RowCursor &rc, uint32_t p, const Span &v) {
+    uint64_t addr = 0;
+    const uint32_t k = rc.at(p, addr);
+    if (k == 16 && rc.stop - p >= 32 && (addr & 31) == 0) {
+        *reinterpret_cast<uint4 *>(addr) = v.a;
+        *reinterpret_cast<uint4 *>(addr + 16) = v.b;
+        return;
+    }
+    if (k) store_bytes(addr, k, v.a);
+    scatter_word(rc, p + 16, v.b);
 }
 
 template <bool kPack>
 __device__ __forceinline__ void tile_fast(const SnapParams &P, const CrcTables &tb, char *chunk,
-                                          const SegRow *rows, int nrows, uint32_t tile0, uint32_t stage_base,
-                                          uint32_t *crc_out) {
+                                          const SegRow *rows, int nrows, uint32_t tile0, uint32_t *crc_out) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t lane4 = lane * 4;
-    const uint32_t wbase = tile0 + warp * kWarpBytes + lane * 16;
-    const uint32_t slot0 = stage_base + (warp * kStages * kRound) + lane * 16;  // this lane's ring
+    const uint32_t wbase = tile0 + warp * kWarpBytes + lane * kLaneSpan;
     const char *nf = reinterpret_cast<const char *>(&tb.NF[0][0][0]);
     RowCursor rc;
     rc.init(rows, 0, nrows, wbase);
-    auto issue = [&](int r) {
-        const uint32_t slot = slot0 + (r % kStages) * kRound;
-        if (kPack)
-            stage_word(rc, wbase + r * kRound, slot);
-        else
-            cp_async16(slot, chunk + wbase + r * kRound);
+    auto load = [&](int r) -> Span {
+        return kPack ? gather_span(rc, wbase + r * kRound) : ld_span(chunk + wbase + r * kRound);
     };
+    Span buf[kAhead + 1];
 #pragma unroll
-    for (int r = 0; r < kStages; ++r) {
-        issue(r);
-        cp_async_commit();
-    }
+    for (int r = 0; r < kAhead; ++r) buf[r] = load(r);
     uint32_t s = 0;
 #pragma unroll
     for (int r = 0; r < kRounds; ++r) {
-        cp_async_wait<kStages - 1>();  // round r's group has landed (one group per round)
-        const uint4 w = lds128(slot0 + (r % kStages) * kRound);
-        if (kPack) st_stream(chunk + wbase + r * kRound, w);
-        s = nib8(nf, lane4, s) ^ raw16(tb, lane4, w);
-        if (!kPack) scatter_word(rc, wbase + r * kRound, w);
-        if (r + kStages < kRounds) issue(r + kStages);
-        cp_async_commit();
+        if (r + kAhead < kRounds) buf[(r + kAhead) % (kAhead + 1)] = load(r + kAhead);
+        Span &w = buf[r % (kAhead + 1)];
+        if (kPack) st_span(chunk + wbase + r * kRound, w);
+        uint4 w0 = w.a;
+        w0.x ^= nib8(nf, lane4, s);  // the register, advanced over the gap, folded into w0
+        s = raw16(tb, lane4, w0);
+        uint4 w1 = w.b;
+        w1.x ^= s;
+        s = raw16(tb, lane4, w1);
+        if (!kPack) scatter_span(rc, wbase + r * kRound, w);
     }
     // lane -> end of this warp's 8 KiB (NL tables), XOR over the warp: the sub-tile's raw CRC
     s = nib8(reinterpret_cast<const char *>(&tb.NL[0][0][0]), lane4, s);
@@ -352,10 +370,8 @@ __device__ __forceinline__ void stage_rows(const SnapParams &P, uint2 tr, SegRow
 
 template <bool kPack>
 __global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
-    // dynamic shared memory: [CrcTables 96 KiB][per-warp cp.async staging rings 96 KiB]
-    extern __shared__ __align__(128) uint8_t smem[];
+    extern __shared__ __align__(128) uint8_t smem[];  // the 96 KiB of CRC tables
     CrcTables &tb = *reinterpret_cast<CrcTables *>(smem);
-    const uint32_t stage_base = (uint32_t)__cvta_generic_to_shared(smem + sizeof(CrcTables));
     __shared__ __align__(16) SegRow srows[2][kMaxTileRows];
     __shared__ uint32_t red[kWarps];
     __shared__ __align__(8) uint64_t tbar;
@@ -381,7 +397,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
         const uint64_t rem = P.chunk_bytes - tile0;
         uint32_t *crc_out = P.tile_crc + ((uint64_t)j * P.tpc + t) * kWarps;
         if (rem >= kTile)
-            tile_fast<kPack>(P, tb, chunk, rows, (int)tr.y, tile0, stage_base, crc_out);
+            tile_fast<kPack>(P, tb, chunk, rows, (int)tr.y, tile0, crc_out);
         else
             tile_generic<kPack>(P, tb, chunk, rows, (int)tr.y, tile0, (uint32_t)rem, crc_out, red);
         __syncthreads();  // srows[buf] and red[] are reused
@@ -489,9 +505,9 @@ static int resident_ctas(int device) {
     if (device < 0 || device >= 64) return 1;
     if (!cached[device]) {
         int per_sm = 0, sms = 0;
-        cudaFuncSetAttribute(k_snapshot<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sizeof(CrcTables) + kStageBytes);
-        cudaFuncSetAttribute(k_snapshot<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sizeof(CrcTables) + kStageBytes);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snapshot<true>, kThreads, sizeof(CrcTables) + kStageBytes);
+        cudaFuncSetAttribute(k_snapshot<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sizeof(CrcTables));
+        cudaFuncSetAttribute(k_snapshot<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sizeof(CrcTables));
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snapshot<true>, kThreads, sizeof(CrcTables));
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
         cached[device] = (per_sm > 0 ? per_sm : 1) * (sms > 0 ? sms : 1);
     }
@@ -507,13 +523,13 @@ int snapshot_grid(int device, uint32_t n_items, uint32_t cap) {
 
 cudaError_t launch_pack(const SnapParams &p, int grid, cudaStream_t s) {
     if (p.count == 0) return cudaSuccess;
-    k_snapshot<true><<<grid, kThreads, sizeof(CrcTables) + kStageBytes, s>>>(p);
+    k_snapshot<true><<<grid, kThreads, sizeof(CrcTables), s>>>(p);
     return cudaGetLastError();
 }
 
 cudaError_t launch_unpack(const SnapParams &p, int grid, cudaStream_t s) {
     if (p.count == 0) return cudaSuccess;
-    k_snapshot<false><<<grid, kThreads, sizeof(CrcTables) + kStageBytes, s>>>(p);
+    k_snapshot<false><<<grid, kThreads, sizeof(CrcTables), s>>>(p);
     return cudaGetLastError();
 }
 

@@ -2,7 +2,7 @@
 # quick K1/K2 iteration: parity tests + microbench + one ncu capture of each
 set -u
 OUT=gpurun_out; mkdir -p $OUT
-timeout 600 python -m pytest tests -m gpu -q -x -p no:cacheprovider 2>&1 | tail -5
+timeout 900 python -m pytest tests -m gpu -q -p no:cacheprovider > $OUT/pytest_gpu.log 2>&1; tail -3 $OUT/pytest_gpu.log
 python tools/k1_bench.py --config c2 --reps 6
 python tools/k1_bench.py --config c2 --reps 6 --unpack
 python tools/k1_bench.py --config c3 --reps 3
