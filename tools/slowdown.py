@@ -15,7 +15,8 @@ import os
 import statistics
 
 
-def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=None):
+def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=None, n_inflight=2, flags=None,
+                   chunk_bytes=64 << 20, writer_threads=4, staging_bytes=0):
     import torch
     import torchvision
 
@@ -40,7 +41,9 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
         state += [p.data, opt.state[p]["momentum_buffer"]]
     shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
     path = path or os.path.join(shm, f"pcc_slowdown_{os.getpid()}.pcc")
-    ck = pcc.PCCheck(path, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.MAPFILE)
+    ck = pcc.PCCheck(path, chunk_bytes=chunk_bytes, max_inflight=n_inflight,
+                     flags=pcc.MAPFILE if flags is None else flags, writer_threads=writer_threads,
+                     staging_bytes=staging_bytes)
     ck.register(state)
 
     def loop(n, checkpoint, it0):
@@ -86,7 +89,7 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
     b, c = statistics.mean(base_t), statistics.mean(ck_t)
     pct = lambda v, q: sorted(v)[min(len(v) - 1, int(q * len(v)))]  # noqa: E731
     return {"model": "vgg16 fp32 SGD(momentum) batch 32, random init, synthetic inputs",
-            "every": every, "iters": iters, "runs": runs,
+            "every": every, "iters": iters, "runs": runs, "N": n_inflight,
             "iter_ms_no_ckpt": b / iters, "iter_ms_ckpt": c / iters,
             "slowdown_pct": (c / b - 1.0) * 100.0,
             "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
