@@ -33,7 +33,7 @@ import numpy as np  # noqa: E402
 METRIC = "snapshot GB/s per GPU & box at 1/2/4/8 B200; % iter slowdown @ ckpt every 10 iters"
 WORKLOADS = {
     "c1": "synthetic 64 MiB fp32 state in 97 mixed-size tensors, 4 MiB chunks, 2 in-flight checkpoints, DRAM-file target",
-    "c2": "VGG-16 fp32 params + SGD momentum (1.107 GB), 64 MiB chunks, 2 in-flight checkpoints, DRAM-file target",
+    "c2": "VGG-16 fp32 params + SGD momentum (1.107 GB), 16 MiB chunks, 2 in-flight checkpoints, DRAM-file target",
     "c3": "OPT-1.3B fp32 params + Adam (15.79 GB), 64 MiB chunks, 4 in-flight checkpoints, DRAM-file target",
     "c4": "BLOOM-7b1 bf16 params + fp32 master + Adam (98.97 GB), 64 MiB chunks, 1/world slice per rank",
 }
@@ -196,6 +196,7 @@ def main():
     ap.add_argument("--config", default="c2")
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
     ap.add_argument("--inflight", type=int, default=2)
+    ap.add_argument("--chunk-mib", type=int, default=0, help="chunk size b in MiB (0 = per-config default)")
     ap.add_argument("--ring-slices", type=int, default=2, help="HBM ring = this many slices")
     ap.add_argument("--no-slowdown", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -220,7 +221,9 @@ def main():
     from synth import config_tensors, make_state
 
     specs = config_tensors(args.config)
-    cb = 4 << 20 if args.config == "c1" else 64 << 20
+    # chunk size b (R2): 4 MiB for the 64 MiB state; 16 MiB for VGG-16 (fig14 sweep: best of
+    # 4/16/64/256 MiB — less zero padding in the last chunk); 64 MiB for the 10-100 GB states
+    cb = args.chunk_mib << 20 if args.chunk_mib else {"c1": 4 << 20, "c2": 16 << 20}.get(args.config, 64 << 20)
     state = make_state(specs, "cuda", seed=0, it=0)
     state_bytes = sum(s.nbytes for s in specs)
     uid = None

@@ -79,7 +79,10 @@ constexpr uint32_t kLaneSpan = 16 * kWpl;            // 32 B
 constexpr uint32_t kRound = 32 * kLaneSpan;          // 1 KiB per warp per round
 constexpr uint32_t kWarpBytes = 8192;                // 8 KiB per warp per tile
 constexpr int kRounds = kWarpBytes / kRound;         // 8
-constexpr int kAhead = 2;                            // rounds loaded ahead of the CRC
+#ifndef PCC_KAHEAD
+#define PCC_KAHEAD 1
+#endif
+constexpr int kAhead = PCC_KAHEAD;                   // rounds loaded ahead of the CRC (A/B builds: -DPCC_KAHEAD)
 constexpr uint32_t kGap = kRound - kLaneSpan;        // zero bytes between a lane's spans
 constexpr uint32_t kTile = kWarps * kWarpBytes;      // 256 KiB per CTA tile
 constexpr int kMaxTileRows = 512;                    // segment rows staged per tile (more -> read from global)

@@ -164,6 +164,7 @@ struct pcc_ctx {
     // per storage slot scratch (a slot belongs to at most one checkpoint in flight)
     std::vector<uint32_t *> tile_crc_dev, crc_dev, scratch_dev;
     std::vector<uint32_t *> crc_host;  // pinned [n + 1] (+ digest)
+    uint32_t *rexpect_dev = nullptr, *rbad_dev = nullptr;  // restore: expected CRCs, bad flags [n]
 
     // HBM ring (Variant B)
     char *ring = nullptr;
@@ -414,6 +415,9 @@ int free_registration(pcc_ctx *c) {
     for (auto p : c->crc_dev) cudaFree(p);
     for (auto p : c->scratch_dev) cudaFree(p);
     for (auto p : c->crc_host) cudaFreeHost(p);
+    cudaFree(c->rexpect_dev);
+    cudaFree(c->rbad_dev);
+    c->rexpect_dev = c->rbad_dev = nullptr;
     c->tile_crc_dev.clear();
     c->crc_dev.clear();
     c->scratch_dev.clear();
@@ -620,6 +624,8 @@ int pcc_register(pcc_ctx *c, const pcc_tensor *t, uint32_t nt) {
         c->scratch_dev.push_back(d);
         c->crc_host.push_back(h);
     }
+    if ((e = cudaMalloc(&c->rexpect_dev, nn * 4)) != cudaSuccess) return cuda_error(e, "restore buffers");
+    if ((e = cudaMalloc(&c->rbad_dev, nn * 4)) != cudaSuccess) return cuda_error(e, "restore buffers");
     // HBM ring: default one whole slice (L139's extra copy)
     if (!c->zerocopy()) {
         uint64_t r = c->cfg.ring_bytes ? c->cfg.ring_bytes / c->cb() : c->n;
@@ -1044,31 +1050,26 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
         return rc;
     }
     HeaderView v = decode_header(hdr, c->sgeom, slot);
-    uint32_t *expect = nullptr, *bad = nullptr, *crc = nullptr, *tile = nullptr, *scr = nullptr;
-    cudaError_t e = cudaSuccess;
-    auto done = [&](int r) {
-        cudaFree(expect);
-        cudaFree(bad);
-        cudaFree(crc);
-        cudaFree(tile);
-        cudaFree(scr);
+    if (!v.ok || !v.layout_ok) {
         std::free(hdr);
-        return r;
-    };
-    if (!v.ok || !v.layout_ok) return done(set_error(PCC_ELAYOUT, "slot header"));
-    if ((e = cudaMalloc(&expect, n * 4)) || (e = cudaMalloc(&bad, n * 4)) || (e = cudaMalloc(&crc, n * 4)) ||
-        (e = cudaMalloc(&tile, n * c->geom.tpc * kWarps * 4)) || (e = cudaMalloc(&scr, 16)))
-        return done(cuda_error(e, "restore buffers"));
-    cudaMemcpy(expect, v.crc, n * 4, cudaMemcpyHostToDevice);
-    cudaMemset(scr, 0, 16);
-    PCC_TRACE("restore: slot %u buffers ready t=%.0f us", slot, c->now_us());
-    // ring for restore: zero-copy mode has none; allocate one batch worth
+        return set_error(PCC_ELAYOUT, "slot header");
+    }
+    // restore runs with nothing in flight (pcc_restore drained): slot 0's scratch is free
+    uint32_t *tile = c->tile_crc_dev[0], *crc = c->crc_dev[0], *scr = c->scratch_dev[0];
+    uint32_t *expect = c->rexpect_dev, *bad = c->rbad_dev;
+    cudaMemcpyAsync(expect, v.crc, n * 4, cudaMemcpyHostToDevice, c->pack_stream);
+    cudaMemsetAsync(scr, 0, 16, c->pack_stream);
+    const uint32_t digest = v.digest;
+    cudaStreamSynchronize(c->pack_stream);  // hdr (the expect source) is freed below
+    std::free(hdr);
+    PCC_TRACE("restore: slot %u header ok t=%.0f us", slot, c->now_us());
+    cudaError_t e = cudaSuccess;
     char *ring = c->ring;
     uint64_t R = c->ring_slots;
     bool own_ring = false;
-    if (!ring) {
+    if (!ring) {  // zero-copy mode keeps no HBM ring
         R = std::min<uint64_t>(n, 16);
-        if ((e = cudaMalloc(&ring, R * cb))) return done(cuda_error(e, "restore ring"));
+        if ((e = cudaMalloc(&ring, R * cb))) return cuda_error(e, "restore ring");
         own_ring = true;
     }
     SnapParams P{};
@@ -1082,32 +1083,36 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     P.tile_crc = tile;
     P.tables = c->tables;
     P.consts = c->consts;
-    cudaEvent_t ev = get_event(c);
+    // batches: H2D of batch b+1 overlaps K2 of batch b when the ring holds the whole slice
+    const bool whole = R >= n;
+    const uint64_t batch = whole ? std::max<uint64_t>(1, (n + 3) / 4) : R;
+    cudaEvent_t ev_copy = get_event(c), ev_k2 = get_event(c);
     const uint64_t data0 = c->slot_data_off(slot);
-    for (uint64_t j0 = 0; j0 < n && rc == PCC_OK; j0 += R) {
-        const uint64_t k = std::min<uint64_t>(R, n - j0);
+    for (uint64_t j0 = 0; j0 < n && rc == PCC_OK; j0 += batch) {
+        const uint64_t k = std::min<uint64_t>(batch, n - j0);
+        if (!whole && j0) cudaStreamWaitEvent(c->copy_stream, ev_k2, 0);  // ring slots reused
         for (uint64_t i = 0; i < k && rc == PCC_OK; ++i) {
-            const char *src;
+            const uint64_t j = j0 + i;
+            char *dst = ring + (whole ? j : i) * cb;
             if (c->mapfile()) {
-                src = c->map + data0 + (j0 + i) * cb;
+                cudaMemcpyAsync(dst, c->map + data0 + j * cb, cb, cudaMemcpyHostToDevice, c->copy_stream);
             } else {  // pread into a pinned staging slot, then H2D (the slot is reused after the copy)
                 char *st = c->staging + (i % c->staging_slots) * cb;
                 if (i >= c->staging_slots) cudaStreamSynchronize(c->copy_stream);
-                rc = pread_full(c->fd, st, cb, data0 + (j0 + i) * cb);
-                src = st;
+                rc = pread_full(c->fd, st, cb, data0 + j * cb);
+                if (rc == PCC_OK) cudaMemcpyAsync(dst, st, cb, cudaMemcpyHostToDevice, c->copy_stream);
             }
-            if (rc == PCC_OK) cudaMemcpyAsync(ring + i * cb, src, cb, cudaMemcpyHostToDevice, c->copy_stream);
         }
-        cudaEventRecord(ev, c->copy_stream);
-        cudaStreamWaitEvent(c->pack_stream, ev, 0);
+        if (!c->mapfile()) cudaStreamSynchronize(c->copy_stream);  // staging reused next batch
+        cudaEventRecord(ev_copy, c->copy_stream);
+        cudaStreamWaitEvent(c->pack_stream, ev_copy, 0);
         P.first = (uint32_t)j0;
         P.count = (uint32_t)k;
-        P.ring_head = (R - j0 % R) % R;
+        P.ring_head = whole ? 0 : (R - j0 % R) % R;
         if ((e = launch_unpack(P, snapshot_grid(c->device, (uint32_t)(k * P.tpc), 0), c->pack_stream)))
             rc = cuda_error(e, "K2");
         c->launches += 1;
-        cudaEventRecord(ev, c->pack_stream);
-        cudaStreamWaitEvent(c->copy_stream, ev, 0);  // next batch's H2D after this K2 read the ring
+        cudaEventRecord(ev_k2, c->pack_stream);
     }
     PCC_TRACE("restore: copies + K2 issued t=%.0f us", c->now_us());
     FinalizeParams F{};
@@ -1132,14 +1137,15 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     }
     cudaStreamSynchronize(c->copy_stream);
     PCC_TRACE("restore: verified t=%.0f us", c->now_us());
-    put_event(c, ev);
+    put_event(c, ev_copy);
+    put_event(c, ev_k2);
     if (own_ring) cudaFree(ring);
-    if (rc) return done(rc);
+    if (rc) return rc;
     for (uint64_t j = 0; j < n; ++j)
         if (flags[j]) bad_out->push_back((uint32_t)(c->first + j));
-    if (!bad_out->empty()) return done(set_error(PCC_ECORRUPT, "chunk CRC32C mismatch"));
-    if (sc[3] != v.digest) return done(set_error(PCC_ECORRUPT, "slice digest mismatch"));
-    return done(PCC_OK);
+    if (!bad_out->empty()) return set_error(PCC_ECORRUPT, "chunk CRC32C mismatch");
+    if (sc[3] != digest) return set_error(PCC_ECORRUPT, "slice digest mismatch");
+    return PCC_OK;
 }
 
 // C3 of SURVEY §2.3: after every rank verified (and scattered) its own slice of iter g, the
