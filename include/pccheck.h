@@ -74,6 +74,10 @@ enum {
                                `world` (packs, persists and commits only its 1/world slice; the
                                global commit reduces over itself).  For measuring one rank's
                                share on one GPU; a restore then covers only this slice. */
+    PCC_SHARDED = 1u << 6,  /* FSDP / ZeRO state (L152 §3.1: "each worker has its own model
+                               shard"): every rank registers its OWN tensors and checkpoints all
+                               of them — no 1/world slicing, no restore fan-out; the global commit
+                               and the restore agreement still run across ranks. */
 };
 
 /* ---- per-checkpoint states (pcc_poll) — SURVEY §8(b) state machine ------------------- */

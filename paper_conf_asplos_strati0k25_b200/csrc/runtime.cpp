@@ -581,7 +581,12 @@ int pcc_register(pcc_ctx *c, const pcc_tensor *t, uint32_t nt) {
     HostLayout full;
     int rc = build_layout(t, nt, c->cfg.align, c->cb(), 0, 0, &full);
     if (rc) return set_error(PCC_EINVAL, "layout");
-    slice_of(full.C, c->cfg.rank, c->cfg.world, &c->first, &c->n);
+    if (c->cfg.flags & PCC_SHARDED) {  // each rank's registration is its own shard: all of it
+        c->first = 0;
+        c->n = full.C;
+    } else {
+        slice_of(full.C, c->cfg.rank, c->cfg.world, &c->first, &c->n);
+    }
     rc = build_layout(t, nt, c->cfg.align, c->cb(), c->first, (int64_t)c->n, &c->layout);
     if (rc) return set_error(PCC_EINVAL, "layout slice");
     build_tile_rows(&c->layout, c->cb(), kTile);
@@ -1294,7 +1299,8 @@ extern "C" int pcc_restore(pcc_ctx *c, uint64_t want_iter, uint32_t flags, uint6
         ops.reduce = [](int64_t *, bool) { return PCC_OK; };
     } else {
         ops.reduce = [c](int64_t *v, bool is_max) { return reduce_i64(c, v, 1, is_max ? NcclComm::kMax : NcclComm::kMin); };
-        if (!(c->cfg.flags & PCC_NOCOMM)) ops.fanout = [c](uint64_t, uint32_t slot) { return dp_fanout(c, slot); };
+        if (!(c->cfg.flags & (PCC_NOCOMM | PCC_SHARDED)))
+            ops.fanout = [c](uint64_t, uint32_t slot) { return dp_fanout(c, slot); };
     }
     ops.verify = [c](uint64_t, uint32_t slot, std::vector<uint32_t> *bad) { return verify_scatter(c, slot, bad); };
     uint64_t it = 0;

@@ -167,3 +167,25 @@ def test_nullsink_and_launch_count(pcc):
         inf = ck.info(h)
         img = oracle.pack([host_bytes(t) for t in ts], 256, 64 << 20)
         assert inf["digest"] == oracle.crc32c(img)
+
+
+def test_sharded_state_checkpoints_whole_registration(pcc, shm):
+    """PCC_SHARDED (FSDP, L152): rank 1 of 2 checkpoints all of its own shard, restores it."""
+    specs = config_tensors("c1")
+    cb = 4 << 20
+    ts = make_state(specs, "cuda", seed=21, it=0)
+    with pcc.PCCheck(shm, chunk_bytes=cb, max_inflight=2, flags=pcc.MAPFILE | pcc.SHARDED | pcc.NOCOMM,
+                     rank=1, world=2) as ck:
+        ck.register(ts)
+        geo = ck.geometry()
+        assert geo["first"] == 0 and geo["count"] == geo["n_chunks"] == 17
+        h = ck.checkpoint(10)
+        ck.wait(h)
+        assert ck.commit() == 10
+        inf = ck.info(h, with_crc=True)
+        img = oracle.pack([host_bytes(t) for t in ts], 256, cb)
+        assert inf["crc"] == [int(x) for x in oracle.chunk_crcs(img, cb)]
+        saved = [host_bytes(t).copy() for t in ts]
+        perturb_state(ts, specs, 21, 5)
+        it, bad = ck.restore()
+        assert it == 10 and all(np.array_equal(host_bytes(t), s) for t, s in zip(ts, saved))
