@@ -87,13 +87,17 @@ constexpr uint32_t kGap = kRound - kLaneSpan;        // zero bytes between a lan
 constexpr uint32_t kTile = kWarps * kWarpBytes;      // 256 KiB per CTA tile
 constexpr int kMaxTileRows = 512;                    // segment rows staged per tile (more -> read from global)
 
-// Shared-memory table block (96 KiB), per-lane replicated nibble tables.
+// Shared-memory table block (160 KiB): 5-bit-indexed tables, replicated once per lane.
+// Entry (table t, value v) of lane l is word (t*32 + v)*32 + l: always bank l.  A 16-byte word
+// is 26 five-bit groups (25 x 5 bits + 3), the 32-bit register 7 groups (6 x 5 + 2).
+constexpr int kG16 = 26;  // 5-bit groups in 128 bits
+constexpr int kG32 = 7;   // 5-bit groups in 32 bits
 struct CrcTables {
-    uint32_t NT[32][16][32];  // NT[q][v][l] = raw16(16-byte word whose nibble q is v, others 0)
-    uint32_t NF[8][16][32];   // NF[q][v][l] = shift(v << 4q, kGap): the zeros before a lane's next span
-    uint32_t NL[8][16][32];   // NL[q][v][l] = shift(v << 4q, kLaneSpan*(31-l)): lane -> warp-region end
+    uint32_t NT[kG16][32][32];  // NT[g][v][l] = raw16(16-byte word whose bits [5g, 5g+5) are v)
+    uint32_t NF[kG32][32][32];  // NF[g][v][l] = shift(v << 5g, kGap): the zeros before a lane's next span
+    uint32_t NL[kG32][32][32];  // NL[g][v][l] = shift(v << 5g, kLaneSpan*(31-l)): lane -> warp-region end
 };
-static_assert(sizeof(CrcTables) == 96 * 1024, "table block size");
+static_assert(sizeof(CrcTables) == 160 * 1024, "table block size");
 
 // Constants that do not need a table.
 struct CrcConsts {
@@ -102,9 +106,6 @@ struct CrcConsts {
     uint32_t x8n_stride;          // x8n(kThreads*16): generic (ragged-tile) path, one thread stride
 };
 
-// XOR of the 8 nibble-table entries selected by the nibbles of x.  `tab` = byte address of
-// table t0 (a shared-memory constant), lane4 = lane*4; entry (t0+k, v) of this lane lives at
-// tab + k*2048 + v*128 + lane4.  ((x >> 4k) & 15) << 7 == (x >> (4k-7)) & 0x780.
 // x >> k as IMAD.HI on the FMA pipe (a plain >> becomes SHF on the ALU pipe, which the
 // LOP3s of the lookups already saturate); mul.hi by a power of two is not strength-reduced.
 __device__ __forceinline__ uint32_t shr_fma(uint32_t x, uint32_t pow2) {
@@ -112,42 +113,67 @@ __device__ __forceinline__ uint32_t shr_fma(uint32_t x, uint32_t pow2) {
     asm("mul.hi.u32 %0, %1, %2;" : "=r"(r) : "r"(x), "r"(pow2));
     return r;
 }
-
-// (a & 0x780) | lane4 as ONE opaque LOP3: written in C the compiler re-associates it into an
+// (hi:lo) >> n, low 32 bits (one SHF)
+__device__ __forceinline__ uint32_t funnel_r(uint32_t lo, uint32_t hi, uint32_t n) {
+    uint32_t r;
+    asm("shf.r.clamp.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(lo), "r"(hi), "r"(n));
+    return r;
+}
+// (a & 0xF80) | lane4 as ONE opaque LOP3: written in C the compiler re-associates it into an
 // AND plus an IADD of a hoisted (table base + lane4) register — one extra instruction per
 // lookup; kept opaque, the table base folds into the LDS's uniform-register + immediate.
-__device__ __forceinline__ uint32_t nib_off(uint32_t a, uint32_t lane4) {
+__device__ __forceinline__ uint32_t grp_off(uint32_t a, uint32_t lane4) {
     uint32_t r;
-    asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(r) : "r"(a), "r"(0x780u), "r"(lane4));
+    asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(r) : "r"(a), "r"(0xF80u), "r"(lane4));
     return r;
 }
 
-__device__ __forceinline__ uint32_t nib8(const char *tab, uint32_t lane4, uint32_t x) {
-    const uint32_t o0 = nib_off(x * 128u, lane4);                 // nibble 0: << 7
-    const uint32_t o1 = nib_off(x * 8u, lane4);                   // nibble 1: << 3
-    const uint32_t o2 = nib_off(shr_fma(x, 1u << 31), lane4);     // nibble k: >> (4k-7)
-    const uint32_t o3 = nib_off(shr_fma(x, 1u << 27), lane4);
-    const uint32_t o4 = nib_off(shr_fma(x, 1u << 23), lane4);
-    const uint32_t o5 = nib_off(shr_fma(x, 1u << 19), lane4);
-    const uint32_t o6 = nib_off(shr_fma(x, 1u << 15), lane4);
-    const uint32_t o7 = nib_off(shr_fma(x, 1u << 11), lane4);
-    const uint32_t a = *reinterpret_cast<const uint32_t *>(tab + 0 * 2048 + o0) ^
-                       *reinterpret_cast<const uint32_t *>(tab + 1 * 2048 + o1) ^
-                       *reinterpret_cast<const uint32_t *>(tab + 2 * 2048 + o2);
-    const uint32_t b = *reinterpret_cast<const uint32_t *>(tab + 3 * 2048 + o3) ^
-                       *reinterpret_cast<const uint32_t *>(tab + 4 * 2048 + o4) ^
-                       *reinterpret_cast<const uint32_t *>(tab + 5 * 2048 + o5);
-    const uint32_t c = *reinterpret_cast<const uint32_t *>(tab + 6 * 2048 + o6) ^
-                       *reinterpret_cast<const uint32_t *>(tab + 7 * 2048 + o7);
-    return a ^ b ^ c;
+// word c of a 128-bit value (compile-time c)
+template <int C>
+__device__ __forceinline__ uint32_t comp(const uint4 &w) {
+    return C == 0 ? w.x : C == 1 ? w.y : C == 2 ? w.z : C == 3 ? w.w : 0u;
 }
 
-// raw16(w): CRC register of the 16 bytes w fed into a zero register (32 nibble lookups).
+// bits [B, B+5) of the little-endian bit string `w`, moved to bits 7..11 (table stride 128 B)
+template <int B>
+__device__ __forceinline__ uint32_t grp_bits(const uint4 &w) {
+    constexpr int wi = B / 32, bi = B % 32;
+    const uint32_t lo = comp<wi>(w);
+    if constexpr (bi <= 7) {
+        return lo * (1u << (7 - bi));  // left shift (IMAD)
+    } else if constexpr (bi <= 27) {
+        return shr_fma(lo, 1u << (39 - bi));  // right shift by bi-7 (IMAD.HI)
+    } else {
+        return funnel_r(lo, comp<wi + 1>(w), bi - 7);  // the group crosses into the next word
+    }
+}
+
+template <int G>
+__device__ __forceinline__ uint32_t lk(const char *tab, uint32_t lane4, const uint4 &w) {
+    return *reinterpret_cast<const uint32_t *>(tab + G * 4096 + grp_off(grp_bits<5 * G>(w), lane4));
+}
+
+// raw16(w): the CRC register of the 16 bytes w fed into a zero register (26 lookups);
 // raw16(w with w.x ^= r) = the register r after absorbing w.
-__device__ __forceinline__ uint32_t raw16(const CrcTables &tb, uint32_t lane4, uint4 w) {
+__device__ __forceinline__ uint32_t raw16(const CrcTables &tb, uint32_t lane4, const uint4 &w) {
     const char *t = reinterpret_cast<const char *>(&tb.NT[0][0][0]);
-    return nib8(t, lane4, w.x) ^ nib8(t + 8 * 2048, lane4, w.y) ^ nib8(t + 16 * 2048, lane4, w.z) ^
-           nib8(t + 24 * 2048, lane4, w.w);
+    uint32_t a = lk<0>(t, lane4, w) ^ lk<1>(t, lane4, w) ^ lk<2>(t, lane4, w);
+    uint32_t b = lk<3>(t, lane4, w) ^ lk<4>(t, lane4, w) ^ lk<5>(t, lane4, w);
+    uint32_t c = lk<6>(t, lane4, w) ^ lk<7>(t, lane4, w) ^ lk<8>(t, lane4, w);
+    uint32_t d = lk<9>(t, lane4, w) ^ lk<10>(t, lane4, w) ^ lk<11>(t, lane4, w);
+    uint32_t e = lk<12>(t, lane4, w) ^ lk<13>(t, lane4, w) ^ lk<14>(t, lane4, w);
+    uint32_t f = lk<15>(t, lane4, w) ^ lk<16>(t, lane4, w) ^ lk<17>(t, lane4, w);
+    uint32_t g = lk<18>(t, lane4, w) ^ lk<19>(t, lane4, w) ^ lk<20>(t, lane4, w);
+    uint32_t h = lk<21>(t, lane4, w) ^ lk<22>(t, lane4, w) ^ lk<23>(t, lane4, w);
+    uint32_t i = lk<24>(t, lane4, w) ^ lk<25>(t, lane4, w);
+    return a ^ b ^ c ^ d ^ e ^ f ^ g ^ h ^ i;
+}
+
+// a 32-bit register through one of the 7-table sets (NF / NL): 7 lookups
+__device__ __forceinline__ uint32_t shift32(const char *tab, uint32_t lane4, uint32_t x) {
+    const uint4 w = make_uint4(x, 0, 0, 0);
+    return lk<0>(tab, lane4, w) ^ lk<1>(tab, lane4, w) ^ lk<2>(tab, lane4, w) ^ lk<3>(tab, lane4, w) ^
+           lk<4>(tab, lane4, w) ^ lk<5>(tab, lane4, w) ^ lk<6>(tab, lane4, w);
 }
 
 }  // namespace pcc

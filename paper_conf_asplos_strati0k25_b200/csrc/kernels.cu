@@ -39,37 +39,44 @@ __device__ uint32_t raw_byte_at(const uint32_t *T0, uint32_t val, int pos) {
 __global__ void k_build_tables(CrcTables *tb, CrcConsts *cs) {
     __shared__ uint32_t x2n[kX2n];
     __shared__ uint32_t T0[256];
-    __shared__ uint32_t vals[48][16];  // distinct entries: NT 32 tables, NF 8, then NL per lane
+    __shared__ uint32_t vals[kG16 + kG32][32];  // distinct entries of NT and NF (NL is per lane)
     const int t = threadIdx.x;  // 256 threads
     if (t == 0) make_x2n(x2n);
     uint32_t r = t;
     for (int k = 0; k < 8; ++k) r = (r & 1u) ? (r >> 1) ^ kPoly : (r >> 1);
     T0[t] = r;
     __syncthreads();
-    // NT: 32 nibble positions x 16 values
-    for (int e = t; e < 32 * 16; e += blockDim.x) {
-        const int q = e >> 4, v = e & 15;
-        vals[q][v] = raw_byte_at(T0, (q & 1) ? (v << 4) : v, q >> 1);
+    // NT: value v at bits [5g, 5g+5) of a 16-byte word (bits past 127 dropped); by linearity the
+    // register is the XOR of its bytes' contributions
+    for (int e = t; e < kG16 * 32; e += blockDim.x) {
+        const int g = e >> 5, v = e & 31, b = 5 * g;
+        uint32_t acc = 0;
+        for (int byte = b / 8; byte <= (b + 4) / 8 && byte < 16; ++byte) {
+            const int sh = b - 8 * byte;  // v's bit 0 sits at bit `sh` of this byte (may be < 0)
+            const uint32_t part = (sh >= 0 ? ((uint32_t)v << sh) : ((uint32_t)v >> -sh)) & 0xFFu;
+            if (part) acc ^= raw_byte_at(T0, part, byte);
+        }
+        vals[g][v] = acc;
     }
     // NF: shift by the gap between a lane's spans
     const uint32_t xr = x8n(x2n, kGap);
-    if (t < 8 * 16) {
-        const int q = t >> 4, v = t & 15;
-        vals[32 + q][v] = multmodp(xr, (uint32_t)v << (4 * q));
+    for (int e = t; e < kG32 * 32; e += blockDim.x) {
+        const int g = e >> 5, v = e & 31;
+        vals[kG16 + g][v] = multmodp(xr, (uint32_t)((uint64_t)v << (5 * g)));
     }
     __syncthreads();
-    for (int e = t; e < 40 * 16 * 32; e += blockDim.x) {
-        const int tab = e / 512, v = (e >> 5) & 15, l = e & 31;
+    for (int e = t; e < (kG16 + kG32) * 32 * 32; e += blockDim.x) {
+        const int tab = e / 1024, v = (e >> 5) & 31, l = e & 31;
         const uint32_t x = vals[tab][v];
-        if (tab < 32)
+        if (tab < kG16)
             tb->NT[tab][v][l] = x;
         else
-            tb->NF[tab - 32][v][l] = x;
+            tb->NF[tab - kG16][v][l] = x;
     }
-    // NL: lane-specific shift 16*(31-l)
-    for (int e = t; e < 8 * 16 * 32; e += blockDim.x) {
-        const int q = e / 512, v = (e >> 5) & 15, l = e & 31;
-        tb->NL[q][v][l] = multmodp(x8n(x2n, kLaneSpan * (31 - l)), (uint32_t)v << (4 * q));
+    // NL: lane-specific shift kLaneSpan*(31-l)
+    for (int e = t; e < kG32 * 32 * 32; e += blockDim.x) {
+        const int g = e / 1024, v = (e >> 5) & 31, l = e & 31;
+        tb->NL[g][v][l] = multmodp(x8n(x2n, kLaneSpan * (31 - l)), (uint32_t)((uint64_t)v << (5 * g)));
     }
     if (t < kX2n) cs->x2n[t] = x2n[t];
     if (t < kWarps) cs->warp_shift[t] = x8n(x2n, (uint64_t)(kWarps - 1 - t) * kWarpBytes);
@@ -274,7 +281,7 @@ __device__ __forceinline__ void tile_fast(const SnapParams &P, const CrcTables &
         Span &w = buf[r % (kAhead + 1)];
         if (kPack) st_span(chunk + wbase + r * kRound, w);
         uint4 w0 = w.a;
-        w0.x ^= nib8(nf, lane4, s);  // the register, advanced over the gap, folded into w0
+        w0.x ^= shift32(nf, lane4, s);  // the register, advanced over the gap, folded into w0
         s = raw16(tb, lane4, w0);
         uint4 w1 = w.b;
         w1.x ^= s;
@@ -282,7 +289,7 @@ __device__ __forceinline__ void tile_fast(const SnapParams &P, const CrcTables &
         if (!kPack) scatter_span(rc, wbase + r * kRound, w);
     }
     // lane -> end of this warp's 8 KiB (NL tables), XOR over the warp: the sub-tile's raw CRC
-    s = nib8(reinterpret_cast<const char *>(&tb.NL[0][0][0]), lane4, s);
+    s = shift32(reinterpret_cast<const char *>(&tb.NL[0][0][0]), lane4, s);
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s ^= __shfl_xor_sync(0xFFFFFFFFu, s, o);
     if (lane == 0) crc_out[warp] = s;
