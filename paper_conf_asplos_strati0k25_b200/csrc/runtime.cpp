@@ -397,8 +397,11 @@ void orchestrate_loop(pcc_ctx *c) {
             c->tasks.push(task);
             ++issued;
         }
-        // chunks never issued (K1 launch failed) count as done so the checkpoint still terminates
+        // chunks never issued (K1 launch failed) count as done so the checkpoint still
+        // terminates, and give their reserved ring chunks back
         const uint32_t unissued = (uint32_t)c->n - issued;
+        if (!c->zerocopy())
+            for (uint32_t j = issued; j < c->n; ++j) ring_release(c, ck->ring_start + j);
         if (c->n == 0 || (unissued && ck->remaining.fetch_sub(unissued) == unissued)) finish_ckpt(c, ck);
     }
 }
