@@ -98,6 +98,15 @@ enum { PCC_U8 = 0, PCC_F32 = 1, PCC_BF16 = 2, PCC_F16 = 3, PCC_F64 = 4, PCC_I64 
 typedef struct pcc_ctx pcc_ctx;
 typedef uint64_t pcc_handle;
 
+/* Caller-supplied collectives (optional, world > 1): when set they replace the library's NCCL
+ * communicator — e.g. a framework that owns its transport, or gloo on CPU.  Both are COLLECTIVE
+ * and called from the thread that called the pcc_* function, in the same order on every rank.
+ *   allreduce: values[count] in place, MAX if is_max else MIN, across all ranks
+ *   allgather: recv[rank * bytes + i] = send_of_rank[i], HOST buffers
+ * Return 0 on success. */
+typedef int (*pcc_allreduce_i64_fn)(void *ctx, int64_t *values, uint32_t count, int is_max);
+typedef int (*pcc_allgather_fn)(void *ctx, const void *send, void *recv, uint64_t bytes_per_rank);
+
 /* Table 2 (L205-L213) configuration parameters, plus placement. */
 typedef struct {
     uint32_t abi_version;      /* PCC_ABI_VERSION                                                  */
@@ -117,6 +126,9 @@ typedef struct {
                                   broadcast by the caller; required when world > 1                 */
     uint32_t align;            /* image alignment of each tensor (R1); 0 = 256                    */
     uint32_t pack_ctas;        /* grid cap for K1 (0 = all SMs); small caps leave SMs to training */
+    pcc_allreduce_i64_fn allreduce; /* optional caller collectives (see above); both or neither */
+    pcc_allgather_fn allgather;
+    void *coll_ctx;
 } pcc_config;
 
 typedef struct {

@@ -37,7 +37,12 @@ class Config(C.Structure):
                 ("max_inflight", C.c_uint32), ("staging_bytes", C.c_uint64), ("ring_bytes", C.c_uint64),
                 ("writer_threads", C.c_uint32), ("flags", C.c_uint32), ("device", C.c_int32), ("rank", C.c_int32),
                 ("world", C.c_int32), ("nccl_unique_id", C.c_void_p), ("align", C.c_uint32),
-                ("pack_ctas", C.c_uint32)]
+                ("pack_ctas", C.c_uint32), ("allreduce", C.c_void_p), ("allgather", C.c_void_p),
+                ("coll_ctx", C.c_void_p)]
+
+
+ALLREDUCE_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.POINTER(C.c_int64), C.c_uint32, C.c_int)
+ALLGATHER_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint64)
 
 
 class Tensor(C.Structure):
@@ -161,13 +166,37 @@ class PCCheck:
 
     def __init__(self, path=None, chunk_bytes=64 << 20, max_inflight=2, staging_bytes=0, ring_bytes=0,
                  writer_threads=4, flags=MAPFILE, device=0, rank=0, world=1, nccl_unique_id=None, align=256,
-                 pack_ctas=0):
+                 pack_ctas=0, allreduce=None, allgather=None):
+        """allreduce(values: list[int], is_max) -> list[int] and allgather(send: bytes) -> bytes
+        (rank-ordered concatenation) replace NCCL when given (e.g. torch.distributed gloo)."""
         self._uid = None
+        self._cbs = None
+        ar = ag = None
+        if allreduce is not None:
+            def _ar(ctx, vals, count, is_max):
+                try:
+                    out = allreduce([int(vals[i]) for i in range(count)], bool(is_max))
+                    for i in range(count):
+                        vals[i] = int(out[i])
+                    return 0
+                except Exception:  # noqa: BLE001
+                    return 1
+
+            def _ag(ctx, send, recv, nbytes):
+                try:
+                    data = allgather(C.string_at(send, nbytes))
+                    C.memmove(recv, data, len(data))
+                    return 0
+                except Exception:  # noqa: BLE001
+                    return 1
+            self._cbs = (ALLREDUCE_FN(_ar), ALLGATHER_FN(_ag))
+            ar, ag = C.cast(self._cbs[0], C.c_void_p), C.cast(self._cbs[1], C.c_void_p)
         if nccl_unique_id is not None:
             self._uid = C.create_string_buffer(bytes(nccl_unique_id), 128)
         self.cfg = Config(ABI_VERSION, path.encode() if path else None, chunk_bytes, max_inflight, staging_bytes,
                           ring_bytes, writer_threads, flags, device, rank, world,
-                          C.cast(self._uid, C.c_void_p) if self._uid is not None else None, align, pack_ctas)
+                          C.cast(self._uid, C.c_void_p) if self._uid is not None else None, align, pack_ctas,
+                          ar, ag, None)
         self._ctx = C.c_void_p()
         _check(_lib.pcc_open(C.byref(self.cfg), C.byref(self._ctx)), "pcc_open")
         self._table = None

@@ -556,7 +556,9 @@ int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
         if (c->fd < 0) return set_errno_error("open checkpoint file", errno);
         c->odirect = flags & O_DIRECT;
     }
-    if (cfg->world > 1 && !(cfg->flags & PCC_NOCOMM)) {
+    if ((cfg->allreduce == nullptr) != (cfg->allgather == nullptr))
+        return set_error(PCC_EINVAL, "allreduce and allgather callbacks go together");
+    if (cfg->world > 1 && !(cfg->flags & PCC_NOCOMM) && !cfg->allreduce) {
         if (!cfg->nccl_unique_id) return set_error(PCC_EINVAL, "nccl_unique_id required for world > 1");
         int rc = c->nccl.init(cfg->nccl_unique_id, cfg->world, cfg->rank);
         if (rc) return rc;
@@ -897,6 +899,9 @@ int pcc_drain(pcc_ctx *c, int64_t timeout_us) {
 // process measuring one rank's share alone) reduces over itself.
 static int reduce_i64(pcc_ctx *c, int64_t *v, size_t n, NcclComm::Op op) {
     if (c->cfg.world == 1 || (c->cfg.flags & PCC_NOCOMM)) return PCC_OK;
+    if (c->cfg.allreduce)
+        return c->cfg.allreduce(c->cfg.coll_ctx, v, (uint32_t)n, op == NcclComm::kMax) ? set_error(PCC_ENCCL, "allreduce callback")
+                                                                                      : PCC_OK;
     return c->nccl.allreduce_i64(v, n, op, c->red_dev, c->red_host, c->aux_stream);
 }
 
@@ -1156,6 +1161,31 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     return PCC_OK;
 }
 
+// allgather of device buffers: NCCL on the library's communicator, or the caller's host
+// callback (staged through pinned host memory)
+static int allgather_dev(pcc_ctx *c, const void *send, void *recv, size_t bytes, cudaStream_t s) {
+    if (!c->cfg.allgather) return c->nccl.allgather(send, recv, bytes, s);
+    const size_t W = (size_t)c->cfg.world;
+    char *hs = nullptr, *hr = nullptr;
+    cudaError_t e;
+    const size_t rbytes = W * bytes;
+    if ((e = cudaMallocHost(&hs, bytes ? bytes : 1)) || (e = cudaMallocHost(&hr, rbytes ? rbytes : 1))) {
+        cudaFreeHost(hs);
+        return cuda_error(e, "allgather staging");
+    }
+    cudaMemcpyAsync(hs, send, bytes, cudaMemcpyDeviceToHost, s);
+    int rc = PCC_OK;
+    if ((e = cudaStreamSynchronize(s))) rc = cuda_error(e, "allgather d2h");
+    if (rc == PCC_OK && c->cfg.allgather(c->cfg.coll_ctx, hs, hr, bytes)) rc = set_error(PCC_ENCCL, "allgather callback");
+    if (rc == PCC_OK) {
+        cudaMemcpyAsync(recv, hr, W * bytes, cudaMemcpyHostToDevice, s);
+        if ((e = cudaStreamSynchronize(s))) rc = cuda_error(e, "allgather h2d");
+    }
+    cudaFreeHost(hs);
+    cudaFreeHost(hr);
+    return rc;
+}
+
 // C3 of SURVEY §2.3: after every rank verified (and scattered) its own slice of iter g, the
 // verified packed chunks cross NVLink with ncclAllGather in groups of G chunks per rank, and
 // each rank K2-verifies + scatters the other ranks' chunks into its registered tensors (the
@@ -1209,7 +1239,7 @@ int dp_fanout(pcc_ctx *c, uint32_t slot) {
         if (rc) return done(rc);
         cudaMemcpy(crc_mine, mine.data(), n_max * 4, cudaMemcpyHostToDevice);
     }
-    if ((rc = c->nccl.allgather(crc_mine, crc_all, n_max * 4, c->pack_stream))) return done(rc);
+    if ((rc = allgather_dev(c, crc_mine, crc_all, n_max * 4, c->pack_stream))) return done(rc);
     const uint64_t data0 = c->slot_data_off(slot);
     std::vector<uint64_t> first_q(W), n_q(W);
     for (uint32_t q = 0; q < W; ++q) slice_of(C, q, W, &first_q[q], &n_q[q]);
@@ -1230,7 +1260,7 @@ int dp_fanout(pcc_ctx *c, uint32_t slot) {
         }
         cudaStreamSynchronize(c->copy_stream);
         if (rc) break;
-        if ((rc = c->nccl.allgather(send, recv, G * cb, c->pack_stream))) break;
+        if ((rc = allgather_dev(c, send, recv, G * cb, c->pack_stream))) break;
         for (uint32_t q = 0; q < W; ++q) {
             if (q == me) continue;
             const uint64_t cnt = n_q[q] > k0 ? std::min<uint64_t>(G, n_q[q] - k0) : 0;
