@@ -610,14 +610,18 @@ int pcc_register(pcc_ctx *c, const pcc_tensor *t, uint32_t nt) {
     if ((e = cudaMalloc(&c->rows_dev, nrows * sizeof(SegRow))) != cudaSuccess) return cuda_error(e, "rows");
     if ((e = cudaMalloc(&c->row_begin_dev, (c->n + 1) * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "rb");
     if (!c->layout.rows.empty())
-        cudaMemcpy(c->rows_dev, c->layout.rows.data(), c->layout.rows.size() * sizeof(SegRow), cudaMemcpyHostToDevice);
-    cudaMemcpy(c->row_begin_dev, c->layout.row_begin.data(), (c->n + 1) * sizeof(uint32_t), cudaMemcpyHostToDevice);
+        cudaMemcpyAsync(c->rows_dev, c->layout.rows.data(), c->layout.rows.size() * sizeof(SegRow),
+                        cudaMemcpyHostToDevice, c->pack_stream);
+    // NB: uploads go on the pack stream, never the legacy stream: a pageable cudaMemcpy may return
+    // before its DMA lands, and the library's streams do not synchronise with the legacy stream
+    cudaMemcpyAsync(c->row_begin_dev, c->layout.row_begin.data(), (c->n + 1) * sizeof(uint32_t), cudaMemcpyHostToDevice,
+                    c->pack_stream);
     {
         const size_t tb = std::max<size_t>(c->layout.tile_rows.size(), 2) * sizeof(uint32_t);
         if ((e = cudaMalloc(&c->tile_rows_dev, tb)) != cudaSuccess) return cuda_error(e, "tile rows");
         if (!c->layout.tile_rows.empty())
-            cudaMemcpy(c->tile_rows_dev, c->layout.tile_rows.data(), c->layout.tile_rows.size() * sizeof(uint32_t),
-                       cudaMemcpyHostToDevice);
+            cudaMemcpyAsync(c->tile_rows_dev, c->layout.tile_rows.data(), c->layout.tile_rows.size() * sizeof(uint32_t),
+                            cudaMemcpyHostToDevice, c->pack_stream);
     }
     if ((e = setup_geometry(&c->geom, c->cb(), (uint32_t)c->n, c->pack_stream)) != cudaSuccess)
         return cuda_error(e, "geometry");
@@ -671,7 +675,8 @@ int pcc_register(pcc_ctx *c, const pcc_tensor *t, uint32_t nt) {
                 cudaSuccess) {
                 munmap(c->map, fbytes);
                 c->map = nullptr;
-                return cuda_error(e, "cudaHostRegister(file mapping)");
+                return cuda_error(e, "cudaHostRegister(file mapping) — PCC_MAPFILE needs a DRAM-backed file "
+                                     "(tmpfs, e.g. /dev/shm); use PWRITE mode (no MAPFILE) for disk files");
             }
             void *dp = nullptr;
             cudaHostGetDevicePointer(&dp, c->map, 0);
@@ -1177,6 +1182,9 @@ static int allgather_dev(pcc_ctx *c, const void *send, void *recv, size_t bytes,
     int rc = PCC_OK;
     if ((e = cudaStreamSynchronize(s))) rc = cuda_error(e, "allgather d2h");
     if (rc == PCC_OK && c->cfg.allgather(c->cfg.coll_ctx, hs, hr, bytes)) rc = set_error(PCC_ENCCL, "allgather callback");
+    PCC_TRACE("allgather: %zu B/rank, sent[0] %08x recv[0] %08x recv[last rank] %08x", bytes,
+              bytes >= 4 ? *reinterpret_cast<uint32_t *>(hs) : 0u, bytes >= 4 ? *reinterpret_cast<uint32_t *>(hr) : 0u,
+              bytes >= 4 ? *reinterpret_cast<uint32_t *>(hr + (W - 1) * bytes) : 0u);
     if (rc == PCC_OK) {
         cudaMemcpyAsync(recv, hr, W * bytes, cudaMemcpyHostToDevice, s);
         if ((e = cudaStreamSynchronize(s))) rc = cuda_error(e, "allgather h2d");
@@ -1224,9 +1232,12 @@ int dp_fanout(pcc_ctx *c, uint32_t slot) {
         (e = cudaMalloc(&crc_all, W * n_max * 4)) || (e = cudaMalloc(&crc_out, C * 4)) || (e = cudaMalloc(&bad, C * 4)) ||
         (e = cudaMalloc(&scr, 16 * W)) || (e = cudaMalloc(&send, G * cb)) || (e = cudaMalloc(&recv, W * G * cb)))
         return done(cuda_error(e, "fanout buffers"));
-    if (!full.rows.empty()) cudaMemcpy(rows, full.rows.data(), full.rows.size() * sizeof(SegRow), cudaMemcpyHostToDevice);
-    cudaMemcpy(rb, full.row_begin.data(), (C + 1) * 4, cudaMemcpyHostToDevice);
-    if (!full.tile_rows.empty()) cudaMemcpy(trows, full.tile_rows.data(), full.tile_rows.size() * 4, cudaMemcpyHostToDevice);
+    cudaStream_t ps = c->pack_stream;  // uploads ordered before the K2 launches on the same stream
+    if (!full.rows.empty())
+        cudaMemcpyAsync(rows, full.rows.data(), full.rows.size() * sizeof(SegRow), cudaMemcpyHostToDevice, ps);
+    cudaMemcpyAsync(rb, full.row_begin.data(), (C + 1) * 4, cudaMemcpyHostToDevice, ps);
+    if (!full.tile_rows.empty())
+        cudaMemcpyAsync(trows, full.tile_rows.data(), full.tile_rows.size() * 4, cudaMemcpyHostToDevice, ps);
     if ((e = setup_geometry(&g2, cb, (uint32_t)n_max, c->pack_stream))) return done(cuda_error(e, "fanout geometry"));
     // this rank's CRC table (from its slot header) -> allgather
     {
@@ -1237,7 +1248,10 @@ int dp_fanout(pcc_ctx *c, uint32_t slot) {
         if (rc == PCC_OK) std::memcpy(mine.data(), hdr + 96, c->n * 4);
         std::free(hdr);
         if (rc) return done(rc);
-        cudaMemcpy(crc_mine, mine.data(), n_max * 4, cudaMemcpyHostToDevice);
+        cudaMemcpyAsync(crc_mine, mine.data(), n_max * 4, cudaMemcpyHostToDevice, c->pack_stream);
+        cudaStreamSynchronize(c->pack_stream);  // `mine` dies at the end of this scope
+        PCC_TRACE("fanout: rank %u slot %u n %llu crc[0] %08x crc[n-1] %08x", me, slot, (unsigned long long)c->n,
+                  mine[0], c->n ? mine[c->n - 1] : 0u);
     }
     if ((rc = allgather_dev(c, crc_mine, crc_all, n_max * 4, c->pack_stream))) return done(rc);
     const uint64_t data0 = c->slot_data_off(slot);
@@ -1304,9 +1318,21 @@ int dp_fanout(pcc_ctx *c, uint32_t slot) {
         }
         if ((e = cudaStreamSynchronize(c->pack_stream))) rc = cuda_error(e, "fanout sync");  // recv reused next group
         std::vector<uint32_t> sc(4 * W);
-        cudaMemcpy(sc.data(), scr, 16 * W, cudaMemcpyDeviceToHost);
-        for (uint32_t q = 0; q < W && rc == PCC_OK; ++q)
-            if (sc[4 * q + 2]) rc = set_error(PCC_ECORRUPT, "chunk corrupted in the NVLink fan-out");
+        cudaMemcpyAsync(sc.data(), scr, 16 * W, cudaMemcpyDeviceToHost, c->pack_stream);
+        cudaStreamSynchronize(c->pack_stream);
+        for (uint32_t q = 0; q < W && rc == PCC_OK; ++q) {
+            if (!sc[4 * q + 2]) continue;
+            if (trace_on()) {
+                const uint64_t cnt = n_q[q] > k0 ? std::min<uint64_t>(G, n_q[q] - k0) : 0;
+                std::vector<uint32_t> got(cnt), exp(cnt);
+                cudaMemcpy(got.data(), crc_out + first_q[q] + k0, cnt * 4, cudaMemcpyDeviceToHost);
+                cudaMemcpy(exp.data(), crc_all + q * n_max + k0, cnt * 4, cudaMemcpyDeviceToHost);
+                for (uint64_t i = 0; i < cnt; ++i)
+                    PCC_TRACE("fanout: rank %u chunk %llu crc %08x expect %08x", q,
+                              (unsigned long long)(first_q[q] + k0 + i), got[i], exp[i]);
+            }
+            rc = set_error(PCC_ECORRUPT, "chunk corrupted in the NVLink fan-out");
+        }
     }
     c->launches += launches;
     return done(rc);
