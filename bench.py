@@ -201,6 +201,9 @@ def main():
     ap.add_argument("--no-slowdown", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--mode", default="mapfile", choices=["mapfile", "zerocopy", "nullsink", "pwrite"])
+    ap.add_argument("--share-gpu", action="store_true", help=argparse.SUPPRESS)  # test hook (see main)
+    ap.add_argument("--collectives", default="torch", choices=["torch", "nccl"],
+                    help="N>1: commit collectives via torch's NCCL process group (callbacks) or the library's own NCCL comm")
     ap.add_argument("--emulate-world", type=int, default=0,
                     help="1 GPU plays rank 0 of this world size alone (PCC_NOCOMM): per-GPU share of a DP job")
     args = ap.parse_args()
@@ -213,10 +216,15 @@ def main():
 
     import torch
     import torch.distributed as dist
+    if args.share_gpu:  # test hook: every rank on cuda:0, gloo transport (NCCL refuses duplicate GPUs)
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.share_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     import paper_conf_asplos_strati0k25_b200 as pcc
     from synth import config_tensors, make_state
 
@@ -227,10 +235,25 @@ def main():
     state = make_state(specs, "cuda", seed=0, it=0)
     state_bytes = sum(s.nbytes for s in specs)
     uid = None
-    if world > 1:
+    coll = {}
+    if world > 1 and args.collectives == "nccl":  # the library's own NCCL communicator
         obj = [pcc.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
+    elif world > 1:  # NCCL through torch's process group, handed to the library as callbacks
+        cdev = "cpu" if args.share_gpu else "cuda"
+
+        def _allreduce(vals, is_max):
+            t = torch.tensor(vals, dtype=torch.int64, device=cdev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX if is_max else dist.ReduceOp.MIN)
+            return t.tolist()
+
+        def _allgather(b):
+            t = torch.frombuffer(bytearray(b), dtype=torch.uint8).to(cdev)
+            parts = [torch.empty_like(t) for _ in range(world)]
+            dist.all_gather(parts, t)
+            return b"".join(x.cpu().numpy().tobytes() for x in parts)
+        coll = dict(allreduce=_allreduce, allgather=_allgather)
     from paper_conf_asplos_strati0k25_b200 import k_layout
     n_est = k_layout([(1 << 20, s.nbytes, s.code) for s in specs], 256, cb)[2]
     slice_est = -(-n_est // world) * cb
@@ -242,7 +265,7 @@ def main():
     shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
     path = None if args.mode == "nullsink" else os.path.join(shm, f"pcc_bench_{os.getpid()}_r{rank}.pcc")
     ck = pcc.PCCheck(path, chunk_bytes=cb, max_inflight=args.inflight, flags=flags, device=local, rank=rank,
-                     world=emu or world, nccl_unique_id=uid, staging_bytes=8 * cb, ring_bytes=args.ring_slices * slice_est)
+                     world=emu or world, nccl_unique_id=uid, **coll, staging_bytes=8 * cb, ring_bytes=args.ring_slices * slice_est)
     ck.register(state)
     geo = ck.geometry()
     slice_bytes = geo["count"] * cb
@@ -268,6 +291,9 @@ def main():
             ck.commit()
         return h
 
+    clocks = ClockSampler(local)  # started before the warm-up so it samples the whole timed region
+    clocks.start()
+    time.sleep(0.5)
     # ---- warm-up
     for _ in range(args.warmup):
         ck.wait(one_ckpt())
@@ -276,8 +302,6 @@ def main():
     barrier()
 
     # ---- timed region: K checkpoints, N in flight
-    clocks = ClockSampler(local)
-    clocks.start()
     launches0 = ck.kernel_launches()
     barrier()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -298,7 +322,7 @@ def main():
     pack_ms = statistics.mean(i["pack_ms"] for i in infos)
     fin_ms = statistics.mean(i["finalize_ms"] for i in infos)
     lat_ms = statistics.median((i["t_committed_us"] - i["t_call_us"]) / 1e3 for i in infos)
-    t = torch.tensor([dev_ms], device="cuda")
+    t = torch.tensor([dev_ms], device="cpu" if args.share_gpu else "cuda")
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms_total = float(t.item())
@@ -332,7 +356,7 @@ def main():
         ck.commit()
     e3.record(stream)
     e3.synchronize()
-    t2 = torch.tensor([e2.elapsed_time(e3)], device="cuda")
+    t2 = torch.tensor([e2.elapsed_time(e3)], device="cpu" if args.share_gpu else "cuda")
     if world > 1:
         dist.all_reduce(t2, op=dist.ReduceOp.MAX)
     e2e_value = state_bytes * e2e_steps / (float(t2.item()) * 1e-3) / 1e9
@@ -383,7 +407,8 @@ def main():
             "config": {"workload": WORKLOADS.get(args.config, args.config), "config": args.config,
                        "state_bytes": state_bytes, "chunk_bytes": cb, "chunks": geo["n_chunks"],
                        "inflight": args.inflight, "mode": args.mode, "hbm_ring_slices": args.ring_slices,
-                       "emulated_rank_of_world": emu or None, "parallelism": f"dp{world}",
+                       "emulated_rank_of_world": emu or None,
+                       "collectives": (args.collectives if world > 1 else None), "parallelism": f"dp{world}",
                        "target": "DRAM file on /dev/shm (tmpfs), mmap + cudaHostRegister" if args.mode != "nullsink"
                        else "null sink", "l2": "inputs larger than L2 (state >> 126 MB)"},
             "per_gpu_gbs": value / world,
