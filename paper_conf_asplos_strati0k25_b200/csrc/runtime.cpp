@@ -97,6 +97,7 @@ struct PersistTask {
     char *dest;  // host address of the chunk (staging slot or file mapping)
     cudaEvent_t ev;
     bool pooled_ev;
+    uint32_t nchunks = 1;  // MAPFILE: chunks [j, j+nchunks) landed by one coalesced copy
 };
 
 template <class T>
@@ -339,7 +340,8 @@ void persist_loop(pcc_ctx *c) {
         PCC_TRACE("persist: ckpt %llu chunk %u landed (%s)", (unsigned long long)ck->t.counter, task.j, cudaGetErrorString(e));
         if (e != cudaSuccess) fail_ckpt(c, task.ck, cuda_error(e, "chunk copy"));
         if (task.pooled_ev) put_event(c, task.ev);
-        if (!c->zerocopy()) ring_release(c, ck->ring_start + task.j);
+        if (!c->zerocopy())
+            for (uint32_t q = 0; q < task.nchunks; ++q) ring_release(c, ck->ring_start + task.j + q);
         const double t = c->now_us();
         if (!c->mapfile()) {
             if (!c->nullsink() && !ck->err.load()) {
@@ -353,7 +355,7 @@ void persist_loop(pcc_ctx *c) {
             ck->t_landed = std::max(ck->t_landed, t);
         }
         PCC_TRACE("persist: ckpt %llu chunk %u done", (unsigned long long)ck->t.counter, task.j);
-        if (ck->remaining.fetch_sub(1) == 1) finish_ckpt(c, task.ck);
+        if (ck->remaining.fetch_sub(task.nchunks) == task.nchunks) finish_ckpt(c, task.ck);
     }
 }
 
@@ -369,7 +371,7 @@ void orchestrate_loop(pcc_ctx *c) {
         }
         size_t li = 0;
         uint32_t issued = 0;
-        for (uint32_t j = 0; j < c->n; ++j) {
+        for (uint32_t j = 0; j < c->n;) {
             Launch L;
             {
                 std::unique_lock<std::mutex> lk(ck->mu);
@@ -384,18 +386,33 @@ void orchestrate_loop(pcc_ctx *c) {
                 task.dest = c->map + c->slot_data_off(ck->t.slot) + (uint64_t)j * c->cb();
             } else {
                 if (j == L.first) cudaStreamWaitEvent(c->copy_stream, L.ev, 0);
-                task.dest = c->mapfile() ? c->map + c->slot_data_off(ck->t.slot) + (uint64_t)j * c->cb()
-                                         : staging_acquire(c);
-                PCC_TRACE("orch: ckpt %llu chunk %u -> %p", (unsigned long long)ck->t.counter, j, (void *)task.dest);
-                const char *src = c->ring + ((ck->ring_start + j) % c->ring_slots) * c->cb();
-                cudaError_t e = cudaMemcpyAsync(task.dest, src, c->cb(), cudaMemcpyDeviceToHost, c->copy_stream);
+                const uint64_t r0 = (ck->ring_start + j) % c->ring_slots;
+                if (c->mapfile()) {
+                    // coalesce chunks of this launch that are contiguous in the ring (and, always,
+                    // in the slot) into one copy of up to kCoalesceBytes: fewer, larger D2H
+                    constexpr uint64_t kCoalesceBytes = 64ull << 20;
+                    uint64_t k = 1;
+                    const uint64_t kmax = std::max<uint64_t>(1, kCoalesceBytes / c->cb());
+                    while (k < kmax && j + k < L.first + L.count && r0 + k < c->ring_slots) ++k;
+                    task.nchunks = (uint32_t)k;
+                    task.dest = c->map + c->slot_data_off(ck->t.slot) + (uint64_t)j * c->cb();
+                } else {
+                    task.dest = staging_acquire(c);
+                }
+                PCC_TRACE("orch: ckpt %llu chunks %u+%u -> %p", (unsigned long long)ck->t.counter, j, task.nchunks,
+                          (void *)task.dest);
+                const char *src = c->ring + r0 * c->cb();
+                cudaError_t e = cudaMemcpyAsync(task.dest, src, task.nchunks * c->cb(), cudaMemcpyDeviceToHost,
+                                                c->copy_stream);
                 if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "D2H"));
                 task.ev = get_event(c);
                 task.pooled_ev = true;
                 cudaEventRecord(task.ev, c->copy_stream);
             }
+            const uint32_t adv = task.nchunks;
             c->tasks.push(task);
-            ++issued;
+            issued += adv;
+            j += adv;
         }
         // chunks never issued (K1 launch failed) count as done so the checkpoint still
         // terminates, and give their reserved ring chunks back
