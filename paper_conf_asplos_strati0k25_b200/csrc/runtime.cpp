@@ -38,6 +38,7 @@
 #include "../../include/pccheck.h"
 #include "commit.hpp"
 #include "errors.hpp"
+#include "fault.hpp"
 #include "kernels.hpp"
 #include "layout.hpp"
 #include "nccl_shim.hpp"
@@ -355,6 +356,7 @@ void persist_loop(pcc_ctx *c) {
             ck->t_landed = std::max(ck->t_landed, t);
         }
         PCC_TRACE("persist: ckpt %llu chunk %u done", (unsigned long long)ck->t.counter, task.j);
+        if (fault_hit("chunk")) fault_die();
         if (ck->remaining.fetch_sub(task.nchunks) == task.nchunks) finish_ckpt(c, task.ck);
     }
 }
