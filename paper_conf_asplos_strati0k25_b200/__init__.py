@@ -172,6 +172,7 @@ class PCCheck:
         self._uid = None
         self._cbs = None
         ar = ag = None
+        cbs = []
         if allreduce is not None:
             def _ar(ctx, vals, count, is_max):
                 try:
@@ -181,7 +182,9 @@ class PCCheck:
                     return 0
                 except Exception:  # noqa: BLE001
                     return 1
-
+            cbs.append(ALLREDUCE_FN(_ar))
+            ar = C.cast(cbs[-1], C.c_void_p)
+        if allgather is not None:
             def _ag(ctx, send, recv, nbytes):
                 try:
                     data = allgather(C.string_at(send, nbytes))
@@ -189,8 +192,9 @@ class PCCheck:
                     return 0
                 except Exception:  # noqa: BLE001
                     return 1
-            self._cbs = (ALLREDUCE_FN(_ar), ALLGATHER_FN(_ag))
-            ar, ag = C.cast(self._cbs[0], C.c_void_p), C.cast(self._cbs[1], C.c_void_p)
+            cbs.append(ALLGATHER_FN(_ag))
+            ag = C.cast(cbs[-1], C.c_void_p)
+        self._cbs = cbs  # the C side holds raw pointers: keep the thunks alive
         if nccl_unique_id is not None:
             self._uid = C.create_string_buffer(bytes(nccl_unique_id), 128)
         self.cfg = Config(ABI_VERSION, path.encode() if path else None, chunk_bytes, max_inflight, staging_bytes,

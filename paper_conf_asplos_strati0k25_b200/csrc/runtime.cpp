@@ -545,6 +545,10 @@ int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
     if ((cfg->flags & PCC_ZEROCOPY) && !(cfg->flags & PCC_MAPFILE))
         return set_error(PCC_EINVAL, "ZEROCOPY needs MAPFILE");
     if (nullsink && (cfg->flags & PCC_MAPFILE)) return set_error(PCC_EINVAL, "NULLSINK excludes MAPFILE");
+    if ((cfg->allreduce == nullptr) != (cfg->allgather == nullptr))
+        return set_error(PCC_EINVAL, "allreduce and allgather callbacks go together");
+    if (cfg->world > 1 && !(cfg->flags & PCC_NOCOMM) && !cfg->allreduce && !cfg->nccl_unique_id)
+        return set_error(PCC_EINVAL, "world > 1 needs nccl_unique_id, caller collectives or PCC_NOCOMM");
     std::unique_ptr<pcc_ctx> c(new pcc_ctx());
     c->cfg = *cfg;
     if (cfg->path) c->path = cfg->path;
@@ -575,10 +579,7 @@ int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
         if (c->fd < 0) return set_errno_error("open checkpoint file", errno);
         c->odirect = flags & O_DIRECT;
     }
-    if ((cfg->allreduce == nullptr) != (cfg->allgather == nullptr))
-        return set_error(PCC_EINVAL, "allreduce and allgather callbacks go together");
     if (cfg->world > 1 && !(cfg->flags & PCC_NOCOMM) && !cfg->allreduce) {
-        if (!cfg->nccl_unique_id) return set_error(PCC_EINVAL, "nccl_unique_id required for world > 1");
         int rc = c->nccl.init(cfg->nccl_unique_id, cfg->world, cfg->rank);
         if (rc) return rc;
         cudaMalloc(&c->red_dev, 4 * sizeof(int64_t));
