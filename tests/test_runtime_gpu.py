@@ -189,3 +189,33 @@ def test_sharded_state_checkpoints_whole_registration(pcc, shm):
         perturb_state(ts, specs, 21, 5)
         it, bad = ck.restore()
         assert it == 10 and all(np.array_equal(host_bytes(t), s) for t, s in zip(ts, saved))
+
+
+def test_edge_cases(pcc, shm):
+    """Empty registration, strictly increasing iters (R5), re-registration of another layout on
+    the same file, waiting with a timeout."""
+    cb = 4 << 20
+    with pcc.PCCheck(shm, chunk_bytes=cb, max_inflight=2, flags=pcc.MAPFILE) as ck:
+        ck.register([])  # nothing registered: C = 0 chunks, the checkpoint still commits
+        h = ck.checkpoint(1)
+        ck.wait(h, timeout_us=10_000_000)
+        assert ck.info(h)["state_name"] == "LOCAL_COMMIT"
+        with pytest.raises(pcc.PCCError) as ei:
+            ck.checkpoint(1)
+        assert ei.value.code == pcc.EORDER
+        specs = config_tensors("c1")[:20]
+        ts = make_state(specs, "cuda", seed=51, it=0)
+        ck.register(ts)  # a different layout on the same file
+        h = ck.checkpoint(5)
+        ck.wait(h)
+        img = oracle.pack([host_bytes(t) for t in ts], 256, cb)
+        assert ck.info(h)["digest"] == oracle.crc32c(img)
+        saved = [host_bytes(t).copy() for t in ts]
+        perturb_state(ts, specs, 51, 3)
+        it, bad = ck.restore()
+        assert it == 5 and all(np.array_equal(host_bytes(t), s) for t, s in zip(ts, saved))
+        # a registration that differs from the newest checkpoint's layout cannot restore it
+        ck.register(ts[:10])
+        with pytest.raises(pcc.PCCError) as ei:
+            ck.restore()
+        assert ei.value.code in (pcc.ELAYOUT, pcc.ENOENT)
