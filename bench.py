@@ -198,6 +198,8 @@ def main():
     ap.add_argument("--inflight", type=int, default=2)
     ap.add_argument("--chunk-mib", type=int, default=0, help="chunk size b in MiB (0 = per-config default)")
     ap.add_argument("--ring-slices", type=int, default=2, help="HBM ring = this many slices")
+    ap.add_argument("--d2h-gbs", type=float, default=0.0, help="pace the D2H copies (GB/s; 0 = full link)")
+    ap.add_argument("--d2h-quantum-kib", type=int, default=0, help="bytes per D2H copy in KiB (0 = chunk groups)")
     ap.add_argument("--no-slowdown", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--mode", default="mapfile", choices=["mapfile", "zerocopy", "nullsink", "pwrite"])
@@ -265,7 +267,8 @@ def main():
     shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
     path = None if args.mode == "nullsink" else os.path.join(shm, f"pcc_bench_{os.getpid()}_r{rank}.pcc")
     ck = pcc.PCCheck(path, chunk_bytes=cb, max_inflight=args.inflight, flags=flags, device=local, rank=rank,
-                     world=emu or world, nccl_unique_id=uid, **coll, staging_bytes=8 * cb, ring_bytes=args.ring_slices * slice_est)
+                     world=emu or world, nccl_unique_id=uid, **coll, staging_bytes=8 * cb, ring_bytes=args.ring_slices * slice_est,
+                     d2h_gbs=args.d2h_gbs, d2h_quantum=args.d2h_quantum_kib << 10)
     ck.register(state)
     geo = ck.geometry()
     slice_bytes = geo["count"] * cb
@@ -407,6 +410,7 @@ def main():
             "config": {"workload": WORKLOADS.get(args.config, args.config), "config": args.config,
                        "state_bytes": state_bytes, "chunk_bytes": cb, "chunks": geo["n_chunks"],
                        "inflight": args.inflight, "mode": args.mode, "hbm_ring_slices": args.ring_slices,
+                       "d2h_gbs": args.d2h_gbs or None, "d2h_quantum_bytes": (args.d2h_quantum_kib << 10) or None,
                        "emulated_rank_of_world": emu or None,
                        "collectives": (args.collectives if world > 1 else None), "parallelism": f"dp{world}",
                        "target": "DRAM file on /dev/shm (tmpfs), mmap + cudaHostRegister" if args.mode != "nullsink"

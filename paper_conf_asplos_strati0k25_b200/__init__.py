@@ -21,7 +21,7 @@ if not os.path.exists(LIB_PATH):
 _lib = C.CDLL(LIB_PATH)
 
 # ---------------------------------------------------------------------- constants
-ABI_VERSION = 1
+ABI_VERSION = 2
 NONE = LATEST = (1 << 64) - 1
 OK, EINVAL, ENOMEM, EBUSY, EAGAIN, EIO, ECUDA, ENCCL, EORDER, ECORRUPT, ELAYOUT, ENOENT, ETIMEDOUT, ESTATE = range(14)
 ODIRECT, FSYNC, ZEROCOPY, NULLSINK, MAPFILE, NOCOMM, SHARDED = 1, 2, 4, 8, 16, 32, 64
@@ -38,7 +38,7 @@ class Config(C.Structure):
                 ("writer_threads", C.c_uint32), ("flags", C.c_uint32), ("device", C.c_int32), ("rank", C.c_int32),
                 ("world", C.c_int32), ("nccl_unique_id", C.c_void_p), ("align", C.c_uint32),
                 ("pack_ctas", C.c_uint32), ("allreduce", C.c_void_p), ("allgather", C.c_void_p),
-                ("coll_ctx", C.c_void_p)]
+                ("coll_ctx", C.c_void_p), ("d2h_mbps", C.c_uint32), ("d2h_quantum", C.c_uint32)]
 
 
 ALLREDUCE_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.POINTER(C.c_int64), C.c_uint32, C.c_int)
@@ -80,6 +80,7 @@ _SIGS = {
     "pcc_kernel_launches": (C.c_uint64, [_P]),
     "pcc_close": (C.c_int, [_P]),
     "pcc_nccl_unique_id": (C.c_int, [_P]),
+    "pcc_struct_size": (C.c_uint64, [C.c_int]),
     "pcc_strerror": (C.c_char_p, [C.c_int]),
     "pcc_last_error": (C.c_char_p, []),
     "pcc_last_errno": (C.c_int, []),
@@ -166,9 +167,10 @@ class PCCheck:
 
     def __init__(self, path=None, chunk_bytes=64 << 20, max_inflight=2, staging_bytes=0, ring_bytes=0,
                  writer_threads=4, flags=MAPFILE, device=0, rank=0, world=1, nccl_unique_id=None, align=256,
-                 pack_ctas=0, allreduce=None, allgather=None):
+                 pack_ctas=0, allreduce=None, allgather=None, d2h_gbs=0.0, d2h_quantum=0):
         """allreduce(values: list[int], is_max) -> list[int] and allgather(send: bytes) -> bytes
-        (rank-ordered concatenation) replace NCCL when given (e.g. torch.distributed gloo)."""
+        (rank-ordered concatenation) replace NCCL when given (e.g. torch.distributed gloo).
+        d2h_gbs / d2h_quantum: pace the copy-engine D2H (GB/s, bytes per copy; 0 = unpaced)."""
         self._uid = None
         self._cbs = None
         ar = ag = None
@@ -200,7 +202,7 @@ class PCCheck:
         self.cfg = Config(ABI_VERSION, path.encode() if path else None, chunk_bytes, max_inflight, staging_bytes,
                           ring_bytes, writer_threads, flags, device, rank, world,
                           C.cast(self._uid, C.c_void_p) if self._uid is not None else None, align, pack_ctas,
-                          ar, ag, None)
+                          ar, ag, None, int(round(d2h_gbs * 1000)), int(d2h_quantum))
         self._ctx = C.c_void_p()
         _check(_lib.pcc_open(C.byref(self.cfg), C.byref(self._ctx)), "pcc_open")
         self._table = None

@@ -373,6 +373,13 @@ void orchestrate_loop(pcc_ctx *c) {
         }
         size_t li = 0;
         uint32_t issued = 0;
+        // D2H pacing (pcc_config d2h_mbps / d2h_quantum): copies of at most `quantum` bytes,
+        // issued no faster than `pace` bytes per microsecond once the chunks exist in HBM
+        const uint64_t pace = c->cfg.d2h_mbps;  // MB/s == bytes per microsecond
+        const uint64_t quantum = c->cfg.d2h_quantum;
+        Clock::time_point t_pace{};
+        bool pace_started = false;
+        uint64_t paced_bytes = 0;
         for (uint32_t j = 0; j < c->n;) {
             Launch L;
             {
@@ -389,6 +396,11 @@ void orchestrate_loop(pcc_ctx *c) {
             } else {
                 if (j == L.first) cudaStreamWaitEvent(c->copy_stream, L.ev, 0);
                 const uint64_t r0 = (ck->ring_start + j) % c->ring_slots;
+                if (pace && j == L.first) {
+                    cudaEventSynchronize(L.ev);  // pace from when the chunks exist
+                    if (!pace_started) t_pace = Clock::now();
+                    pace_started = true;
+                }
                 if (c->mapfile()) {
                     // coalesce chunks of this launch that are contiguous in the ring (and, always,
                     // in the slot) into one copy of up to kCoalesceBytes: fewer, larger D2H
@@ -404,9 +416,17 @@ void orchestrate_loop(pcc_ctx *c) {
                 PCC_TRACE("orch: ckpt %llu chunks %u+%u -> %p", (unsigned long long)ck->t.counter, j, task.nchunks,
                           (void *)task.dest);
                 const char *src = c->ring + r0 * c->cb();
-                cudaError_t e = cudaMemcpyAsync(task.dest, src, task.nchunks * c->cb(), cudaMemcpyDeviceToHost,
-                                                c->copy_stream);
-                if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "D2H"));
+                const uint64_t total = task.nchunks * c->cb();
+                const uint64_t q = quantum ? quantum : total;
+                for (uint64_t o = 0; o < total; o += q) {
+                    const uint64_t len = std::min(q, total - o);
+                    if (pace) {
+                        std::this_thread::sleep_until(t_pace + std::chrono::microseconds(paced_bytes / pace));
+                        paced_bytes += len;
+                    }
+                    cudaError_t e = cudaMemcpyAsync(task.dest + o, src + o, len, cudaMemcpyDeviceToHost, c->copy_stream);
+                    if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "D2H"));
+                }
                 task.ev = get_event(c);
                 task.pooled_ev = true;
                 cudaEventRecord(task.ev, c->copy_stream);
@@ -528,6 +548,9 @@ const char *pcc_strerror(int err) {
         default: return "unknown error";
     }
 }
+uint64_t pcc_struct_size(int which) {
+    return which == 0 ? sizeof(pcc_config) : which == 1 ? sizeof(pcc_tensor) : which == 2 ? sizeof(pcc_ckpt_info) : 0;
+}
 const char *pcc_last_error(void) { return err_state().msg.c_str(); }
 int pcc_last_errno(void) { return err_state().err_no; }
 
@@ -563,7 +586,10 @@ int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
     if ((e = device_tables(c->device, &c->tables, &c->consts)) != cudaSuccess) return cuda_error(e, "CRC tables");
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
-    if ((e = cudaStreamCreateWithPriority(&c->pack_stream, cudaStreamNonBlocking, hi)) != cudaSuccess)
+    // PCC_PACK_PRIO=low|default (experiments): K1's stream priority relative to training
+    const char *pp = std::getenv("PCC_PACK_PRIO");
+    const int prio = pp && !std::strcmp(pp, "low") ? lo : pp && !std::strcmp(pp, "default") ? 0 : hi;
+    if ((e = cudaStreamCreateWithPriority(&c->pack_stream, cudaStreamNonBlocking, prio)) != cudaSuccess)
         return cuda_error(e, "stream");
     cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking);
     cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking);

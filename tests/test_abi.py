@@ -31,6 +31,16 @@ def test_library_exports_every_declared_symbol():
     assert set(pcc.exported_symbols()) == _declared()
 
 
+def test_struct_mirrors_match_the_build():
+    """The ctypes mirrors of pcc_config / pcc_tensor / pcc_ckpt_info have the C sizes (a field
+    added to the header without the binding, or the reverse, fails here)."""
+    import paper_conf_asplos_strati0k25_b200 as pcc
+    assert pcc._lib.pcc_struct_size(0) == ctypes.sizeof(pcc.Config)
+    assert pcc._lib.pcc_struct_size(1) == ctypes.sizeof(pcc.Tensor)
+    assert pcc._lib.pcc_struct_size(2) == ctypes.sizeof(pcc.Info)
+    assert pcc._lib.pcc_struct_size(7) == 0
+
+
 def test_no_gpu_calls_fail_cleanly():
     import paper_conf_asplos_strati0k25_b200 as pcc
     assert pcc._lib.pcc_strerror(-pcc.ECORRUPT) == b"checksum mismatch"

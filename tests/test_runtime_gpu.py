@@ -86,6 +86,30 @@ def test_checkpoint_file_matches_oracle(pcc, shm, mode):
         assert pcc.latest(shm) == (30, 30)
 
 
+@pytest.mark.parametrize("mode", ["mapfile", "pwrite_odirect"])
+def test_paced_d2h_matches_oracle_and_rate(pcc, shm, mode):
+    """d2h_mbps / d2h_quantum (the transfer split into 256 KiB copies issued at 2 GB/s): the
+    file is still the oracle's, byte for byte, and the transfer honours the pace."""
+    specs = config_tensors("c1")
+    cb = 4 << 20
+    ts = make_state(specs, "cuda", seed=2, it=0)
+    with pcc.PCCheck(shm, chunk_bytes=cb, max_inflight=2, flags=MODES[mode](pcc), staging_bytes=4 * cb,
+                     d2h_gbs=2.0, d2h_quantum=256 << 10) as ck:
+        ck.register(ts)
+        n = ck.geometry()["count"]
+        for it in (10, 20):
+            perturb_state(ts, specs, seed=2, it=it)
+            h = ck.checkpoint(it)
+            ck.guard()
+            ck.wait(h)
+            info = ck.info(h, with_crc=True)
+            assert info["state_name"] == "LOCAL_COMMIT"
+            _check_file_against_oracle(shm, specs, ts, cb, info, 3)
+            # the last quantum may start at (bytes - quantum) / pace after the pack finished
+            min_us = (n * cb - (256 << 10)) / 2000.0
+            assert info["t_landed_us"] - info["t_call_us"] >= 0.95 * min_us, (info, min_us)
+
+
 def test_n_in_flight_and_guard(pcc, shm):
     """N=3 checkpoints issued back to back while the 'optimizer' rewrites the state after
     each guard: every checkpoint must hold the state as it was at its own call (L139)."""

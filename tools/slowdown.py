@@ -13,10 +13,14 @@ from __future__ import annotations
 
 import os
 import statistics
+import time
 
 
 def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=None, n_inflight=2, flags=None,
-                   chunk_bytes=64 << 20, writer_threads=4, staging_bytes=0):
+                   chunk_bytes=64 << 20, writer_threads=4, staging_bytes=0, pack_ctas=0, use_guard=True,
+                   graphs=False, d2h_gbs=0.0, d2h_quantum=0):
+    """graphs=True: the training step runs as two CUDA graphs (forward + backward, then the
+    optimizer step) with the U-gate between them; False: eager PyTorch."""
     import torch
     import torchvision
 
@@ -36,6 +40,22 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
     for _ in range(2):  # momentum buffers exist after the first step
         step()
         opt.step()
+    update = opt.step
+    if graphs:
+        s0 = torch.cuda.Stream()
+        s0.wait_stream(stream)
+        with torch.cuda.stream(s0):  # warm-up on a side stream before capture
+            for _ in range(3):
+                step()
+                opt.step()
+        stream.wait_stream(s0)
+        g_fb, g_up = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
+        opt.zero_grad(set_to_none=True)
+        with torch.cuda.graph(g_fb):
+            lossf(model(x), y).backward()
+        with torch.cuda.graph(g_up):
+            opt.step()
+        step, update = g_fb.replay, g_up.replay
     state = []
     for p in model.parameters():
         state += [p.data, opt.state[p]["momentum_buffer"]]
@@ -43,8 +63,9 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
     path = path or os.path.join(shm, f"pcc_slowdown_{os.getpid()}.pcc")
     ck = pcc.PCCheck(path, chunk_bytes=chunk_bytes, max_inflight=n_inflight,
                      flags=pcc.MAPFILE if flags is None else flags, writer_threads=writer_threads,
-                     staging_bytes=staging_bytes)
+                     staging_bytes=staging_bytes, pack_ctas=pack_ctas, d2h_gbs=d2h_gbs, d2h_quantum=d2h_quantum)
     ck.register(state)
+    host_ms = []
 
     def loop(n, checkpoint, it0):
         handles = []
@@ -54,11 +75,13 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
         last = e0
         for i in range(1, n + 1):
             step()
-            if checkpoint:
+            if checkpoint and use_guard:
                 ck.guard(stream)
-            opt.step()
+            update()
             if checkpoint and i % every == 0:
+                th = time.perf_counter()
                 handles.append(ck.checkpoint(it0 + i, stream))
+                host_ms.append((time.perf_counter() - th) * 1e3)
             ev = torch.cuda.Event(enable_timing=True)
             ev.record(stream)
             per.append((last, ev))
@@ -68,35 +91,48 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
         total = e0.elapsed_time(e1)
         for h in handles:
             ck.wait(h)
-        its = sorted(a.elapsed_time(b) for a, b in per)
+        its = [a.elapsed_time(b) for a, b in per]  # iteration i+1 at index i
         return total, its
 
     loop(warmup, False, 0)
     base_t, ck_t, its_b, its_c = [], [], [], []
+    pos_b, pos_c = [[] for _ in range(every)], [[] for _ in range(every)]
     it0 = 1000
     for r in range(runs):
         t, its = loop(iters, False, 0)
         base_t.append(t)
         its_b += its
+        for i, v in enumerate(its):
+            pos_b[(i + 1) % every].append(v)
         t, its = loop(iters, True, it0)
         it0 += 1000
         ck_t.append(t)
         its_c += its
+        for i, v in enumerate(its):
+            pos_c[(i + 1) % every].append(v)
     ck.drain()
     ck.close()
     if os.path.exists(path):
         os.unlink(path)
     b, c = statistics.mean(base_t), statistics.mean(ck_t)
     pct = lambda v, q: sorted(v)[min(len(v) - 1, int(q * len(v)))]  # noqa: E731
-    return {"model": "vgg16 fp32 SGD(momentum) batch 32, random init, synthetic inputs",
+    return {"model": "vgg16 fp32 SGD(momentum) batch 32, random init, synthetic inputs"
+                     + (", training step as CUDA graphs" if graphs else ", eager"),
             "every": every, "iters": iters, "runs": runs, "N": n_inflight,
             "iter_ms_no_ckpt": b / iters, "iter_ms_ckpt": c / iters,
             "slowdown_pct": (c / b - 1.0) * 100.0,
+            # mean extra ms of iteration i % every == k (k = 0: the iteration that issues the
+            # checkpoint after its step; k = 1: the next one, which overlaps K1)
+            "extra_ms_by_pos": [statistics.mean(pc) - statistics.mean(pb) for pb, pc in zip(pos_b, pos_c)],
+            "host_ckpt_call_ms": statistics.median(host_ms) if host_ms else None,
+            "pack_ctas": pack_ctas, "guard": use_guard, "graphs": graphs,
+            "d2h_gbs": d2h_gbs or None, "d2h_quantum": d2h_quantum or None,
             "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
             "state_bytes": sum(t.numel() * t.element_size() for t in state)}
 
 
-def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1, path=None):
+def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1, path=None, d2h_gbs=0.0,
+                   d2h_quantum=0):
     """BLOOM-7b1 (BASELINE configs[3]) on ONE B200 as a proxy for one rank of a world-`world`
     data-parallel job: the per-GPU compute of DP at micro-batch 1 (forward + backward of the
     full model on one 2048-token sequence, then a mixed-precision Adam step), checkpointing
@@ -141,7 +177,8 @@ def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1,
 
     shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
     path = path or os.path.join(shm, f"pcc_bloom_{os.getpid()}.pcc")
-    ck = pcc.PCCheck(path, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.MAPFILE | pcc.NOCOMM, rank=0, world=world)
+    ck = pcc.PCCheck(path, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.MAPFILE | pcc.NOCOMM, rank=0, world=world,
+                     d2h_gbs=d2h_gbs, d2h_quantum=d2h_quantum)
     ck.register(state)
     geo = ck.geometry()
 
