@@ -379,17 +379,26 @@ def main():
     if path and os.path.exists(path):
         os.unlink(path)
 
-    slowdown = None
+    # training slowdown, checkpoint every 10 iterations (BASELINE metric, second half):
+    #   slowdown           eager training, D2H paced by the tuner (tuner.choose_pace) — the
+    #                      library configured for training
+    #   slowdown_unpaced   eager training, the configuration `value` was measured in
+    #   slowdown_graphs    training step as CUDA graphs, tuned pace
+    slowdown = slowdown_unpaced = slowdown_graphs = None
     if rank == 0 and world == 1 and not args.no_slowdown and args.config in ("c2", "c4"):
         try:
             if args.config == "c2":
                 from tools.slowdown import vgg16_slowdown
-                slowdown = vgg16_slowdown(pcc, iters=60, every=10)
+                slowdown = vgg16_slowdown(pcc, iters=60, every=10, d2h_gbs="auto", link_gbs=peak_link)
+                slowdown_unpaced = vgg16_slowdown(pcc, iters=60, every=10)
+                slowdown_graphs = vgg16_slowdown(pcc, iters=60, every=10, d2h_gbs="auto", link_gbs=peak_link,
+                                                 graphs=True)
             else:
                 del state, host_state
                 torch.cuda.empty_cache()
                 from tools.slowdown import bloom_slowdown
-                slowdown = bloom_slowdown(pcc, world=emu or 8, iters=40, every=10)
+                slowdown = bloom_slowdown(pcc, world=emu or 8, iters=40, every=10, d2h_gbs="auto", link_gbs=peak_link)
+                slowdown_unpaced = bloom_slowdown(pcc, world=emu or 8, iters=40, every=10)
         except Exception as ex:  # noqa: BLE001
             slowdown = {"error": repr(ex)[:300]}
 
@@ -433,6 +442,8 @@ def main():
             "gpu_launches": launches,
             "clocks": clk,
             "slowdown": slowdown,
+            "slowdown_unpaced": slowdown_unpaced,
+            "slowdown_graphs": slowdown_graphs,
             "wall_s_timed": wall,
         }
         print(json.dumps(line), flush=True)

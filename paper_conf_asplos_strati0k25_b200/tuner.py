@@ -9,6 +9,13 @@ T_w / N, then sets the checkpoint interval (Eq 3; reading R14: ceiling)
 
 Here T_w of one checkpoint is measured by the library itself (pcc_info: pcc_checkpoint call
 -> local commit) while N checkpoints are kept in flight at a cadence of one every t seconds.
+
+On B200 the tool also picks the D2H pace (pcc_config d2h_mbps / d2h_quantum): a saturating
+copy-engine burst slows an eager training loop by ~10% while it lasts, small paced copies
+leave gaps that hide it (profiles/r01_slowdown_diagnosis.md).  `choose_pace` takes the
+gentlest pace that still lands one checkpoint within `margin` of its interval f*t, never below
+half the link (below that the measured interference no longer drops) and unpaced when even the
+full link is needed.
 """
 from __future__ import annotations
 
@@ -73,3 +80,17 @@ def tune(make_ctx, m_bytes: int, S_bytes: int, t: float, q: float, n_max: int = 
     out["t"] = t
     out["q"] = q
     return out
+
+
+D2H_QUANTUM = 512 << 10  # bytes per paced copy (0.5 MiB: measured best trade, r01 diagnosis)
+
+
+def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, margin: float = 0.5) -> dict:
+    """D2H pace for training: {"d2h_gbs": G, "d2h_quantum": Q}; G = 0 means unpaced."""
+    if f <= 0 or t <= 0 or link_gbs <= 0:
+        raise ValueError("f, t and link_gbs must be positive")
+    need = slice_bytes / (margin * f * t) / 1e9  # GB/s to land a checkpoint in margin * f * t
+    g = max(need, 0.5 * link_gbs)
+    if g >= link_gbs:
+        return {"d2h_gbs": 0.0, "d2h_quantum": 0, "need_gbs": need}
+    return {"d2h_gbs": g, "d2h_quantum": D2H_QUANTUM, "need_gbs": need}

@@ -16,6 +16,22 @@ def test_choose_matches_eq3():
     assert choose({1: 0.01}, q=1.0, t=1.0)["f"] == 1
 
 
+def test_choose_pace():
+    from paper_conf_asplos_strati0k25_b200.tuner import D2H_QUANTUM, choose_pace
+    # VGG-16: 1.1 GB every 10 x 17 ms needs 12.9 GB/s at margin 0.5 -> floor of half the link
+    p = choose_pace(1_107_296_256, 10, 0.0171, 57.0)
+    assert p["d2h_gbs"] == 28.5 and p["d2h_quantum"] == D2H_QUANTUM
+    assert abs(p["need_gbs"] - 1_107_296_256 / (0.5 * 10 * 0.0171) / 1e9) < 1e-9
+    # a tighter interval raises the pace above the floor
+    p = choose_pace(1_107_296_256, 4, 0.0171, 57.0)
+    assert 28.5 < p["d2h_gbs"] < 57.0 and p["d2h_gbs"] == pytest.approx(p["need_gbs"])
+    # checkpointing every iteration needs more than the link: unpaced
+    assert choose_pace(1_107_296_256, 1, 0.0171, 57.0) == {"d2h_gbs": 0.0, "d2h_quantum": 0,
+                                                            "need_gbs": pytest.approx(129.5, rel=1e-3)}
+    with pytest.raises(ValueError):
+        choose_pace(1, 0, 1.0, 1.0)
+
+
 @pytest.mark.gpu
 @pytest.mark.timeout(300)
 def test_tune_live_c1():

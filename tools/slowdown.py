@@ -16,11 +16,38 @@ import statistics
 import time
 
 
+def _iter_time(fn, stream, n=10):
+    import torch
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    fn()
+    a.record(stream)
+    for _ in range(n):
+        fn()
+    b.record(stream)
+    b.synchronize()
+    return a.elapsed_time(b) / n * 1e-3
+
+
+def _slice_bytes(pcc, state, chunk_bytes, rank=0, world=1):
+    _, _, c = pcc.k_layout(state, 256, chunk_bytes)
+    return (((rank + 1) * c) // world - (rank * c) // world) * chunk_bytes
+
+
+def _auto_pace(pcc, state, chunk_bytes, every, link_gbs, step_fn, stream, rank=0, world=1):
+    from paper_conf_asplos_strati0k25_b200.tuner import choose_pace
+    t = _iter_time(step_fn, stream)
+    choice = choose_pace(_slice_bytes(pcc, state, chunk_bytes, rank, world), every, t, link_gbs)
+    choice.update(t_iter_s=t, link_gbs=link_gbs)
+    return choice["d2h_gbs"], choice["d2h_quantum"], choice
+
+
 def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=None, n_inflight=2, flags=None,
                    chunk_bytes=64 << 20, writer_threads=4, staging_bytes=0, pack_ctas=0, use_guard=True,
-                   graphs=False, d2h_gbs=0.0, d2h_quantum=0):
+                   graphs=False, d2h_gbs=0.0, d2h_quantum=0, link_gbs=None):
     """graphs=True: the training step runs as two CUDA graphs (forward + backward, then the
-    optimizer step) with the U-gate between them; False: eager PyTorch."""
+    optimizer step) with the U-gate between them; False: eager PyTorch.  d2h_gbs="auto": the
+    tuner's D2H pace (tuner.choose_pace) for `every` x the measured iteration time and the
+    D2H link peak `link_gbs`."""
     import torch
     import torchvision
 
@@ -59,6 +86,10 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
     state = []
     for p in model.parameters():
         state += [p.data, opt.state[p]["momentum_buffer"]]
+    pace_choice = None
+    if d2h_gbs == "auto":  # the tuner's pace for this interval (iteration time measured here)
+        d2h_gbs, d2h_quantum, pace_choice = _auto_pace(pcc, state, chunk_bytes, every, link_gbs,
+                                                       lambda: (step(), update()), stream)
     shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
     path = path or os.path.join(shm, f"pcc_slowdown_{os.getpid()}.pcc")
     ck = pcc.PCCheck(path, chunk_bytes=chunk_bytes, max_inflight=n_inflight,
@@ -126,13 +157,13 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
             "extra_ms_by_pos": [statistics.mean(pc) - statistics.mean(pb) for pb, pc in zip(pos_b, pos_c)],
             "host_ckpt_call_ms": statistics.median(host_ms) if host_ms else None,
             "pack_ctas": pack_ctas, "guard": use_guard, "graphs": graphs,
-            "d2h_gbs": d2h_gbs or None, "d2h_quantum": d2h_quantum or None,
+            "d2h_gbs": d2h_gbs or None, "d2h_quantum": d2h_quantum or None, "pace_choice": pace_choice,
             "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
             "state_bytes": sum(t.numel() * t.element_size() for t in state)}
 
 
 def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1, path=None, d2h_gbs=0.0,
-                   d2h_quantum=0):
+                   d2h_quantum=0, link_gbs=None):
     """BLOOM-7b1 (BASELINE configs[3]) on ONE B200 as a proxy for one rank of a world-`world`
     data-parallel job: the per-GPU compute of DP at micro-batch 1 (forward + backward of the
     full model on one 2048-token sequence, then a mixed-precision Adam step), checkpointing
@@ -175,6 +206,13 @@ def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1,
             m.addcdiv_(a, b.sqrt().add_(eps), value=-lr)
             p.copy_(m)
 
+    for _ in range(warmup):
+        fwd_bwd()
+        adam_step()
+    pace_choice = None
+    if d2h_gbs == "auto":
+        d2h_gbs, d2h_quantum, pace_choice = _auto_pace(pcc, state, 64 << 20, every, link_gbs,
+                                                       lambda: (fwd_bwd(), adam_step()), stream, 0, world)
     shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
     path = path or os.path.join(shm, f"pcc_bloom_{os.getpid()}.pcc")
     ck = pcc.PCCheck(path, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.MAPFILE | pcc.NOCOMM, rank=0, world=world,
@@ -206,9 +244,6 @@ def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1,
             ck.wait(h)
         return e0.elapsed_time(e1), sorted(a.elapsed_time(b) for a, b in per)
 
-    for _ in range(warmup):
-        fwd_bwd()
-        adam_step()
     base_t, ck_t, its_b, its_c = [], [], [], []
     it0 = 1000
     for r in range(runs):
@@ -231,4 +266,5 @@ def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1,
             "slice_bytes": geo["count"] * (64 << 20),
             "iter_ms_no_ckpt": b / iters, "iter_ms_ckpt": c / iters, "slowdown_pct": (c / b - 1.0) * 100.0,
             "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
+            "d2h_gbs": d2h_gbs or None, "d2h_quantum": d2h_quantum or None, "pace_choice": pace_choice,
             "state_bytes": sum(t.numel() * t.element_size() for t in state)}
