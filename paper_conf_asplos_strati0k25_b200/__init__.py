@@ -285,6 +285,34 @@ class PCCheck:
             pass
 
 
+_STATE_KEYS = ("momentum_buffer", "exp_avg", "exp_avg_sq", "step")
+
+
+def state_tensors(optimizer, masters=None):
+    """The registration list of reading R11 for a torch optimizer: per parameter
+    in param-group order ``[param, (fp32 master), momentum_buffer | exp_avg, exp_avg_sq, step]``.
+    ``masters`` maps a parameter to its fp32 master copy (mixed precision).  Returns
+    ``(tensors, names)``; a state entry that is not a tensor (or lives on the host, e.g. the
+    CPU ``step`` of non-fused Adam) raises — every registered tensor must be device memory."""
+    import torch
+    tensors, names = [], []
+    k = 0
+    for g in optimizer.param_groups:
+        for p in g["params"]:
+            entries = [("param", p.data)]
+            if masters is not None and p in masters:
+                entries.append(("master", masters[p]))
+            st = optimizer.state.get(p, {})
+            entries += [(key, st[key]) for key in _STATE_KEYS if key in st]
+            for key, t in entries:
+                if not isinstance(t, torch.Tensor) or (t.device.type != p.device.type):
+                    raise ValueError(f"param {k} {key}: not a tensor on {p.device} (use fused/capturable optimizers)")
+                tensors.append(t)
+                names.append(f"{k}.{key}")
+            k += 1
+    return tensors, names
+
+
 def latest(path):
     g, l = C.c_uint64(), C.c_uint64()
     rc = _lib.pcc_latest(path.encode(), C.byref(g), C.byref(l))

@@ -72,7 +72,10 @@ __host__ __device__ inline uint32_t x8n(const uint32_t *x2n, uint64_t n) {
 // therefore conflict-free (1 wavefront), at 36 lookups per 16 bytes.  (Byte-indexed
 // slicing-by-16 tables cost 20 lookups per 16 B, but random indices collide in banks ~2.9-way
 // on average; ncu showed the L1/shared pipe at 81% with that design, K1 at 0.45 of HBM.)
-constexpr int kWarps = 32;
+#ifndef PCC_KWARPS
+#define PCC_KWARPS 32
+#endif
+constexpr int kWarps = PCC_KWARPS;                   // warps per CTA (A/B builds: -DPCC_KWARPS)
 constexpr int kThreads = kWarps * 32;
 constexpr int kWpl = 2;                              // 16-byte words per lane per round
 constexpr uint32_t kLaneSpan = 16 * kWpl;            // 32 B

@@ -3,6 +3,6 @@
 set -u
 for v in paper_conf_asplos_strati0k25_b200 build/va*; do
   echo "== $v"
-  PCC_LIB=$v/libpccheck.so python tools/k1_bench.py --config c2 --reps 8
+  PCC_LIB=$v/libpccheck.so python tools/k1_bench.py --config c2 --cb 16777216 --reps 8
   PCC_LIB=$v/libpccheck.so python tools/k1_bench.py --config c3 --reps 4
 done
