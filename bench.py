@@ -117,23 +117,49 @@ def d2h_peak_gbs(torch, nbytes=1 << 30):
     return nbytes / (best * 1e-3) / 1e9
 
 
-def cpu_baseline(specs, state, cb, budget_bytes=2 << 30):
-    """The oracle as it stands (single-threaded plain C: byte-loop pack + byte-at-a-time CRC32C)
-    on a bounded sample: one pack call over the first chunks of the same image, up to
-    `budget_bytes` (the whole image for VGG-16), then the per-chunk CRCs."""
+def cpu_baseline(specs, state, cb, budget_bytes=2 << 30, threads=1, hb=None):
+    """The oracle as it stands (plain C: byte-loop pack + byte-at-a-time CRC32C) on a bounded
+    sample: pack calls over the first chunks of the same image, up to `budget_bytes` (the whole
+    image for VGG-16), then the per-chunk CRCs.  threads > 1: that many host threads over
+    disjoint chunk ranges (K independent oracles; ctypes drops the GIL)."""
     import oracle
+    from concurrent.futures import ThreadPoolExecutor
     from synth import host_bytes
-    hb = [host_bytes(t) for t in state]
+    hb = hb if hb is not None else [host_bytes(t) for t in state]
     nb = [s.nbytes for s in specs]
     off, end, c = oracle.layout(nb, 256, cb)
     k = max(1, min(c, budget_bytes // cb))
+    parts = [(i * k // threads, (i + 1) * k // threads) for i in range(threads)]
+    parts = [(a, b) for a, b in parts if b > a]
+
+    def run(ab):
+        if threads == 1:
+            img = oracle.pack(hb, 256, cb, first_chunk=ab[0], count=ab[1] - ab[0])
+        else:  # an independent oracle per range, handed only the tensors overlapping it
+            lo, hi = ab[0] * cb, ab[1] * cb
+            mine = {i: hb[i] for i in range(len(nb)) if int(off[i]) < hi and int(off[i]) + nb[i] > lo and nb[i]}
+            img = oracle.pack_chunks_sparse(nb, mine, 256, cb, ab[0], ab[1] - ab[0])
+        oracle.chunk_crcs(img, cb)
+
     t0 = time.perf_counter()
-    img = oracle.pack(hb, 256, cb, first_chunk=0, count=k)
-    oracle.chunk_crcs(img, cb)
+    with ThreadPoolExecutor(len(parts)) as ex:
+        list(ex.map(run, parts))
     dt = time.perf_counter() - t0
-    return {"value": k * cb / dt / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle",
+    return {"value": k * cb / dt / 1e9, "unit": "GB/s", "cores": len(parts), "kind": "oracle",
             "sample": f"pack + CRC32C of chunks 0..{k - 1} of {c} ({cb >> 20} MiB) of the same image "
-                      f"({k * cb / 1e9:.3f} GB, {dt:.1f} s, single-threaded plain C)"}
+                      f"({k * cb / 1e9:.3f} GB, {dt:.1f} s, plain C, {len(parts)} thread(s) over disjoint chunk ranges)",
+            "cpu": _cpu_model(), "nproc": os.cpu_count()}
+
+
+def _cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
 
 
 def load_traffic(name):
@@ -408,9 +434,12 @@ def main():
         k1_bytes = 2 * slice_bytes  # read the slice's state bytes + write the packed slice (R3: pads count)
         k1_achieved = k1_bytes / (pack_ms * 1e-3) / 1e9
         link_achieved = slice_bytes / (ms_total * 1e-3 / args.steps) / 1e9
-        cpu = None
+        cpu = cpu_all = None
         if not args.no_cpu_baseline and args.config in ("c1", "c2", "c3"):
-            cpu = cpu_baseline(specs, state, cb)
+            from synth import host_bytes
+            hb = [host_bytes(t) for t in state]
+            cpu = cpu_baseline(specs, state, cb, hb=hb)
+            cpu_all = cpu_baseline(specs, state, cb, hb=hb, threads=len(os.sched_getaffinity(0)))
         line = {
             "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_total / args.steps, "higher_is_better": True,
@@ -437,6 +466,7 @@ def main():
             "finalize_ms": fin_ms,
             "restore": restore,
             "cpu_baseline": cpu,
+            "cpu_baseline_all_cores": cpu_all,
             "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": h2d_bytes,
                     "d2h_bytes_per_step": slice_bytes + 4 * (geo["count"] + 1)},
             "gpu_launches": launches,
