@@ -57,21 +57,25 @@ __host__ __device__ inline uint32_t x8n(const uint32_t *x2n, uint64_t n) {
 }
 
 // ---------------------------------------------------------------- kernel geometry
-// One CTA of 32 warps per SM (all warps share one 96 KiB copy of the tables), tile = 256 KiB
-// of one chunk, warp region = 8 KiB = 8 rounds of 1 KiB.  In round r lane l owns the 32 bytes
-// at warp_base + r*1024 + 32*l: one 256-bit load and one 256-bit store per lane, so every warp
+// One CTA of 32 warps per SM (all warps share one copy of the tables), tile = 256 KiB of one
+// chunk, warp region = 8 KiB = 8 rounds of 1 KiB.  In round r lane l owns the 32 bytes at
+// warp_base + r*1024 + 32*l: one 256-bit load and one 256-bit store per lane, so every warp
 // access is 1 KiB contiguous.  Loads run kAhead rounds ahead in registers.  Per round:
 //     x = shift(s, 992);  s = raw16(w0 ^ x);  s = raw16(w1 ^ s)
 // (feeding a 16-byte word into register r equals raw16 of the word with its first 4 bytes
-// XOR r).  After the last round a lane's register is shifted to its warp-region end
-// (shift by 32*(31-l)) and XOR-reduced over the warp: one raw CRC per 8 KiB sub-tile; the
-// finalize kernel folds sub-tiles, chunks and the slice digest.
+// XOR r).  After the last round every lane writes its register (relative to the end of its
+// last span) to global memory; the finalize kernel shifts each lane to its warp-region end
+// (NL tables, shift by 32*(31-l)), XORs a warp's 32 lanes into the 8 KiB sub-tile's raw CRC and
+// folds sub-tiles, chunks and the slice digest.
 //
-// Lookups are NIBBLE tables replicated once per lane: entry (table t, nibble v) of lane l
-// sits at word (t*16 + v)*32 + l, i.e. always in bank l.  Every shared load of the CRC is
-// therefore conflict-free (1 wavefront), at 36 lookups per 16 bytes.  (Byte-indexed
-// slicing-by-16 tables cost 20 lookups per 16 B, but random indices collide in banks ~2.9-way
-// on average; ncu showed the L1/shared pipe at 81% with that design, K1 at 0.45 of HBM.)
+// Lookups are tables replicated once per lane: entry (table t, value v) of lane l sits at
+// word (t*V + v)*32 + l, i.e. always in bank l, so every shared load of the CRC is
+// conflict-free (1 wavefront).  NT (the 16-byte word -> register map) is indexed by
+// kNtBits-bit groups: 6 bits = 22 lookups per 16 B in 169 KiB; NF (the 992-byte gap shift of
+// the register) by 5-bit groups, 7 lookups in 24.5 KiB.  A last group narrower than the others
+// gets a table of only its own 2^bits values.  (Byte-indexed slicing-by-16 tables cost 20
+// lookups per 16 B, but random indices collide in banks ~2.9-way on average; ncu showed the
+// L1/shared pipe at 81% with that design, K1 at 0.45 of HBM.)
 #ifndef PCC_KWARPS
 #define PCC_KWARPS 32
 #endif
@@ -89,18 +93,31 @@ constexpr int kAhead = PCC_KAHEAD;                   // rounds loaded ahead of t
 constexpr uint32_t kGap = kRound - kLaneSpan;        // zero bytes between a lane's spans
 constexpr uint32_t kTile = kWarps * kWarpBytes;      // 256 KiB per CTA tile
 constexpr int kMaxTileRows = 512;                    // segment rows staged per tile (more -> read from global)
+constexpr int kLaneOut = 32;                         // raw CRCs K1/K2 write per warp sub-tile (one per lane)
 
-// Shared-memory table block (160 KiB): 5-bit-indexed tables, replicated once per lane.
-// Entry (table t, value v) of lane l is word (t*32 + v)*32 + l: always bank l.  A 16-byte word
-// is 26 five-bit groups (25 x 5 bits + 3), the 32-bit register 7 groups (6 x 5 + 2).
-constexpr int kG16 = 26;  // 5-bit groups in 128 bits
-constexpr int kG32 = 7;   // 5-bit groups in 32 bits
+#ifndef PCC_NTBITS
+#define PCC_NTBITS 6
+#endif
+constexpr int kNtBits = PCC_NTBITS;                  // NT group width (A/B builds: -DPCC_NTBITS=5)
+constexpr int kNtVals = 1 << kNtBits;
+constexpr int kG16 = (128 + kNtBits - 1) / kNtBits;  // groups in a 16-byte word: 22 (6-bit) / 26 (5-bit)
+constexpr int kNtLastBits = 128 - (kG16 - 1) * kNtBits;
+constexpr int kG32 = 7;                              // 5-bit groups in the 32-bit register (6 x 5 + 2)
+constexpr uint32_t kNtTab = kNtVals * 128;           // bytes per full NT table (V values x 32 lanes x 4 B)
+constexpr uint32_t kNtBytes = (kG16 - 1) * kNtTab + (1u << kNtLastBits) * 128;
+constexpr uint32_t kRegTab = 32 * 128;               // bytes per full NF / NL table
+constexpr uint32_t kRegBytes = (kG32 - 1) * kRegTab + (1u << 2) * 128;
+
+// Table block.  K1/K2 load NT + NF (the first kK1TableBytes) into shared memory; NL is read by
+// the finalize kernel only.  Word index of entry (t, v, l): t*V*32 + v*32 + l inside each part.
 struct CrcTables {
-    uint32_t NT[kG16][32][32];  // NT[g][v][l] = raw16(16-byte word whose bits [5g, 5g+5) are v)
-    uint32_t NF[kG32][32][32];  // NF[g][v][l] = shift(v << 5g, kGap): the zeros before a lane's next span
-    uint32_t NL[kG32][32][32];  // NL[g][v][l] = shift(v << 5g, kLaneSpan*(31-l)): lane -> warp-region end
+    uint32_t NT[kNtBytes / 4];   // NT[t][v][l] = raw16(16-byte word whose bits [kNtBits*t, +kNtBits) are v)
+    uint32_t NF[kRegBytes / 4];  // NF[g][v][l] = shift(v << 5g, kGap): the zeros before a lane's next span
+    uint32_t NL[kRegBytes / 4];  // NL[g][v][l] = shift(v << 5g, kLaneSpan*(31-l)): lane -> warp-region end
 };
-static_assert(sizeof(CrcTables) == 160 * 1024, "table block size");
+constexpr uint32_t kK1TableBytes = kNtBytes + kRegBytes;
+static_assert(kK1TableBytes % 16 == 0, "TMA bulk copy size");
+static_assert(kK1TableBytes + 2 * kMaxTileRows * 16 + 1024 <= 227 * 1024, "K1 shared memory");
 
 // Constants that do not need a table.
 struct CrcConsts {
@@ -122,12 +139,13 @@ __device__ __forceinline__ uint32_t funnel_r(uint32_t lo, uint32_t hi, uint32_t 
     asm("shf.r.clamp.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(lo), "r"(hi), "r"(n));
     return r;
 }
-// (a & 0xF80) | lane4 as ONE opaque LOP3: written in C the compiler re-associates it into an
+// (a & mask) | lane4 as ONE opaque LOP3: written in C the compiler re-associates it into an
 // AND plus an IADD of a hoisted (table base + lane4) register — one extra instruction per
 // lookup; kept opaque, the table base folds into the LDS's uniform-register + immediate.
+template <uint32_t kMask>
 __device__ __forceinline__ uint32_t grp_off(uint32_t a, uint32_t lane4) {
     uint32_t r;
-    asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(r) : "r"(a), "r"(0xF80u), "r"(lane4));
+    asm("lop3.b32 %0, %1, %2, %3, 0xEA;" : "=r"(r) : "r"(a), "r"(kMask), "r"(lane4));
     return r;
 }
 
@@ -137,46 +155,56 @@ __device__ __forceinline__ uint32_t comp(const uint4 &w) {
     return C == 0 ? w.x : C == 1 ? w.y : C == 2 ? w.z : C == 3 ? w.w : 0u;
 }
 
-// bits [B, B+5) of the little-endian bit string `w`, moved to bits 7..11 (table stride 128 B)
-template <int B>
+// bits [B, B+W) of the little-endian bit string `w`, moved to bits 7.. (table stride 128 B);
+// higher garbage bits are masked by grp_off
+template <int B, int W>
 __device__ __forceinline__ uint32_t grp_bits(const uint4 &w) {
     constexpr int wi = B / 32, bi = B % 32;
     const uint32_t lo = comp<wi>(w);
     if constexpr (bi <= 7) {
         return lo * (1u << (7 - bi));  // left shift (IMAD)
-    } else if constexpr (bi <= 27) {
+    } else if constexpr (bi + W <= 32) {
         return shr_fma(lo, 1u << (39 - bi));  // right shift by bi-7 (IMAD.HI)
     } else {
         return funnel_r(lo, comp<wi + 1>(w), bi - 7);  // the group crosses into the next word
     }
 }
 
-template <int G>
+// entry of table G (groups of W bits, tables of kTab bytes) for the group's value in `w`
+template <int G, int W, uint32_t kTab>
 __device__ __forceinline__ uint32_t lk(const char *tab, uint32_t lane4, const uint4 &w) {
-    return *reinterpret_cast<const uint32_t *>(tab + G * 4096 + grp_off(grp_bits<5 * G>(w), lane4));
+    constexpr uint32_t kMask = ((1u << W) - 1u) << 7;
+    return *reinterpret_cast<const uint32_t *>(tab + G * kTab + grp_off<kMask>(grp_bits<W * G, W>(w), lane4));
 }
 
-// raw16(w): the CRC register of the 16 bytes w fed into a zero register (26 lookups);
-// raw16(w with w.x ^= r) = the register r after absorbing w.
-__device__ __forceinline__ uint32_t raw16(const CrcTables &tb, uint32_t lane4, const uint4 &w) {
-    const char *t = reinterpret_cast<const char *>(&tb.NT[0][0][0]);
-    uint32_t a = lk<0>(t, lane4, w) ^ lk<1>(t, lane4, w) ^ lk<2>(t, lane4, w);
-    uint32_t b = lk<3>(t, lane4, w) ^ lk<4>(t, lane4, w) ^ lk<5>(t, lane4, w);
-    uint32_t c = lk<6>(t, lane4, w) ^ lk<7>(t, lane4, w) ^ lk<8>(t, lane4, w);
-    uint32_t d = lk<9>(t, lane4, w) ^ lk<10>(t, lane4, w) ^ lk<11>(t, lane4, w);
-    uint32_t e = lk<12>(t, lane4, w) ^ lk<13>(t, lane4, w) ^ lk<14>(t, lane4, w);
-    uint32_t f = lk<15>(t, lane4, w) ^ lk<16>(t, lane4, w) ^ lk<17>(t, lane4, w);
-    uint32_t g = lk<18>(t, lane4, w) ^ lk<19>(t, lane4, w) ^ lk<20>(t, lane4, w);
-    uint32_t h = lk<21>(t, lane4, w) ^ lk<22>(t, lane4, w) ^ lk<23>(t, lane4, w);
-    uint32_t i = lk<24>(t, lane4, w) ^ lk<25>(t, lane4, w);
+template <int G>
+__device__ __forceinline__ uint32_t nt(const char *t, uint32_t lane4, const uint4 &w) {
+    if constexpr (G < kG16) return lk<G, kNtBits, kNtTab>(t, lane4, w);
+    else return 0u;
+}
+
+// raw16(w): the CRC register of the 16 bytes w fed into a zero register (kG16 lookups);
+// raw16(w with w.x ^= r) = the register r after absorbing w.  XOR tree in 3-input LOP3s.
+__device__ __forceinline__ uint32_t raw16(const char *t, uint32_t lane4, const uint4 &w) {
+    uint32_t a = nt<0>(t, lane4, w) ^ nt<1>(t, lane4, w) ^ nt<2>(t, lane4, w);
+    uint32_t b = nt<3>(t, lane4, w) ^ nt<4>(t, lane4, w) ^ nt<5>(t, lane4, w);
+    uint32_t c = nt<6>(t, lane4, w) ^ nt<7>(t, lane4, w) ^ nt<8>(t, lane4, w);
+    uint32_t d = nt<9>(t, lane4, w) ^ nt<10>(t, lane4, w) ^ nt<11>(t, lane4, w);
+    uint32_t e = nt<12>(t, lane4, w) ^ nt<13>(t, lane4, w) ^ nt<14>(t, lane4, w);
+    uint32_t f = nt<15>(t, lane4, w) ^ nt<16>(t, lane4, w) ^ nt<17>(t, lane4, w);
+    uint32_t g = nt<18>(t, lane4, w) ^ nt<19>(t, lane4, w) ^ nt<20>(t, lane4, w);
+    uint32_t h = nt<21>(t, lane4, w) ^ nt<22>(t, lane4, w) ^ nt<23>(t, lane4, w);
+    uint32_t i = nt<24>(t, lane4, w) ^ nt<25>(t, lane4, w);
+    static_assert(kG16 <= 26, "raw16 unrolls at most 26 groups");
     return a ^ b ^ c ^ d ^ e ^ f ^ g ^ h ^ i;
 }
 
-// a 32-bit register through one of the 7-table sets (NF / NL): 7 lookups
+// a 32-bit register through one of the 7-table (5-bit) sets NF / NL: 7 lookups
 __device__ __forceinline__ uint32_t shift32(const char *tab, uint32_t lane4, uint32_t x) {
     const uint4 w = make_uint4(x, 0, 0, 0);
-    return lk<0>(tab, lane4, w) ^ lk<1>(tab, lane4, w) ^ lk<2>(tab, lane4, w) ^ lk<3>(tab, lane4, w) ^
-           lk<4>(tab, lane4, w) ^ lk<5>(tab, lane4, w) ^ lk<6>(tab, lane4, w);
+    return lk<0, 5, kRegTab>(tab, lane4, w) ^ lk<1, 5, kRegTab>(tab, lane4, w) ^ lk<2, 5, kRegTab>(tab, lane4, w) ^
+           lk<3, 5, kRegTab>(tab, lane4, w) ^ lk<4, 5, kRegTab>(tab, lane4, w) ^ lk<5, 5, kRegTab>(tab, lane4, w) ^
+           lk<6, 5, kRegTab>(tab, lane4, w);
 }
 
 }  // namespace pcc

@@ -49,7 +49,7 @@ int prepare(const pcc_tensor *t, uint32_t n, uint32_t align, uint64_t cb, uint64
     const size_t nrows = L->rows.size() ? L->rows.size() : 1;
     if ((e = cudaMalloc(&S->rows, nrows * sizeof(SegRow))) != cudaSuccess) return cuda_error(e, "rows");
     if ((e = cudaMalloc(&S->row_begin, (count + 1) * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "rb");
-    if ((e = cudaMalloc(&S->tile_crc, count * S->geom.tpc * kWarps * sizeof(uint32_t))) != cudaSuccess)
+    if ((e = cudaMalloc(&S->tile_crc, count * tile_crc_words(S->geom.tpc) * sizeof(uint32_t))) != cudaSuccess)
         return cuda_error(e, "tile crc");
     if ((e = cudaMalloc(&S->tile_rows, L->tile_rows.size() * sizeof(uint32_t))) != cudaSuccess)
         return cuda_error(e, "tile rows");
@@ -106,6 +106,7 @@ extern "C" int pcc_k_pack(const pcc_tensor *t, uint32_t n, uint32_t align, uint6
     if (e != cudaSuccess) return cuda_error(e, "K1 launch");
     FinalizeParams F{};
     F.tile_crc = S.tile_crc;
+    F.tables = P.tables;
     F.n = (uint32_t)count;
     F.tpc = P.tpc;
     F.tile_shift = S.geom.tile_shift;
@@ -137,6 +138,7 @@ extern "C" int pcc_k_unpack(const pcc_tensor *t, uint32_t n, uint32_t align, uin
     if (e != cudaSuccess) return cuda_error(e, "K2 launch");
     FinalizeParams F{};
     F.tile_crc = S.tile_crc;
+    F.tables = P.tables;
     F.n = (uint32_t)count;
     F.tpc = P.tpc;
     F.tile_shift = S.geom.tile_shift;

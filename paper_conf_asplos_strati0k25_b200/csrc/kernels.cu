@@ -9,16 +9,16 @@
 // moved verbatim, so NaN payloads / denormals survive (R1).
 //
 // Execution model:
-//   * one CTA = 8 warps processes 32 KiB tiles of one chunk, grid-stride over
-//     (chunk, tile) items; grid = SMs x resident CTAs (or the pack_ctas cap);
-//   * in each of 8 rounds a warp moves 512 contiguous bytes: every lane one 16-B
-//     vector (ld.global.nc.v4 / st.global.cs.v4) — all 8 rounds are loaded before any
-//     CRC work so 8 x 16 B per lane are in flight;
-//   * the segment-table row under each word is tracked by a per-lane cursor; a 16-B word
-//     holds bytes of at most one row because rows start 16-B aligned in the chunk;
-//   * CRC: per-lane register, advanced by the gap table and slicing-by-16 (20 shared
-//     memory lookups per 16 B), 5-level shuffle tree, warp combine with x8n constants;
-//     tile CRCs go to global memory and k_finalize folds tiles -> chunk -> slice digest.
+//   * one CTA of 32 warps per SM (the tables fill its shared memory), tile = 256 KiB of one
+//     chunk, grid-stride over (chunk, tile) items; grid = SMs (or the pack_ctas cap);
+//   * a warp owns 8 KiB of the tile = 8 rounds of 1 KiB: lane l moves the 32 bytes at
+//     32*l with one 256-bit load and one 256-bit store, one round of loads ahead;
+//   * the segment-table row under each word is tracked by a per-lane cursor over the tile's
+//     rows (staged in shared memory by cp.async); a 16-B word holds bytes of at most one row
+//     because rows start 16-B aligned in the chunk;
+//   * CRC (crc32c.cuh): per-lane register, advanced over the gap by the NF tables and fed the
+//     words through the 6-bit NT tables (51 conflict-free LDS per 32 B); every lane writes its
+//     register, and k_finalize folds lanes -> 8 KiB sub-tiles -> chunks -> slice digest.
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <mutex>
@@ -39,44 +39,43 @@ __device__ uint32_t raw_byte_at(const uint32_t *T0, uint32_t val, int pos) {
 __global__ void k_build_tables(CrcTables *tb, CrcConsts *cs) {
     __shared__ uint32_t x2n[kX2n];
     __shared__ uint32_t T0[256];
-    __shared__ uint32_t vals[kG16 + kG32][32];  // distinct entries of NT and NF (NL is per lane)
+    __shared__ uint32_t vt[kG16][kNtVals];  // distinct NT entries (all lanes share them)
+    __shared__ uint32_t vf[kG32][32];       // distinct NF entries (NL is per lane)
     const int t = threadIdx.x;  // 256 threads
     if (t == 0) make_x2n(x2n);
     uint32_t r = t;
     for (int k = 0; k < 8; ++k) r = (r & 1u) ? (r >> 1) ^ kPoly : (r >> 1);
     T0[t] = r;
     __syncthreads();
-    // NT: value v at bits [5g, 5g+5) of a 16-byte word (bits past 127 dropped); by linearity the
-    // register is the XOR of its bytes' contributions
-    for (int e = t; e < kG16 * 32; e += blockDim.x) {
-        const int g = e >> 5, v = e & 31, b = 5 * g;
+    // NT: value v at bits [kNtBits*g, +kNtBits) of a 16-byte word (bits past 127 dropped); by
+    // linearity the register is the XOR of its bytes' contributions
+    for (int e = t; e < kG16 * kNtVals; e += blockDim.x) {
+        const int g = e / kNtVals, v = e % kNtVals, b = kNtBits * g;
         uint32_t acc = 0;
-        for (int byte = b / 8; byte <= (b + 4) / 8 && byte < 16; ++byte) {
+        for (int byte = b / 8; byte <= (b + kNtBits - 1) / 8 && byte < 16; ++byte) {
             const int sh = b - 8 * byte;  // v's bit 0 sits at bit `sh` of this byte (may be < 0)
             const uint32_t part = (sh >= 0 ? ((uint32_t)v << sh) : ((uint32_t)v >> -sh)) & 0xFFu;
             if (part) acc ^= raw_byte_at(T0, part, byte);
         }
-        vals[g][v] = acc;
+        vt[g][v] = acc;
     }
     // NF: shift by the gap between a lane's spans
     const uint32_t xr = x8n(x2n, kGap);
     for (int e = t; e < kG32 * 32; e += blockDim.x) {
         const int g = e >> 5, v = e & 31;
-        vals[kG16 + g][v] = multmodp(xr, (uint32_t)((uint64_t)v << (5 * g)));
+        vf[g][v] = multmodp(xr, (uint32_t)((uint64_t)v << (5 * g)));
     }
     __syncthreads();
-    for (int e = t; e < (kG16 + kG32) * 32 * 32; e += blockDim.x) {
-        const int tab = e / 1024, v = (e >> 5) & 31, l = e & 31;
-        const uint32_t x = vals[tab][v];
-        if (tab < kG16)
-            tb->NT[tab][v][l] = x;
-        else
-            tb->NF[tab - kG16][v][l] = x;
+    // replicate per lane; the last table of each set holds only its group's 2^bits values
+    for (uint32_t e = t; e < kNtBytes / 4; e += blockDim.x) {
+        const uint32_t g = e / (kNtVals * 32), v = (e / 32) % kNtVals;
+        tb->NT[e] = vt[g][v];
     }
-    // NL: lane-specific shift kLaneSpan*(31-l)
-    for (int e = t; e < kG32 * 32 * 32; e += blockDim.x) {
-        const int g = e / 1024, v = (e >> 5) & 31, l = e & 31;
-        tb->NL[g][v][l] = multmodp(x8n(x2n, kLaneSpan * (31 - l)), (uint32_t)((uint64_t)v << (5 * g)));
+    for (uint32_t e = t; e < kRegBytes / 4; e += blockDim.x) {
+        const uint32_t g = e >> 10, v = (e >> 5) & 31, l = e & 31;
+        tb->NF[e] = vf[g][v];
+        // NL: lane-specific shift kLaneSpan*(31-l)
+        tb->NL[e] = multmodp(x8n(x2n, kLaneSpan * (31 - l)), (uint32_t)((uint64_t)v << (5 * g)));
     }
     if (t < kX2n) cs->x2n[t] = x2n[t];
     if (t < kWarps) cs->warp_shift[t] = x8n(x2n, (uint64_t)(kWarps - 1 - t) * kWarpBytes);
@@ -260,12 +259,11 @@ __device__ __forceinline__ void scatter_span(RowCursor &rc, uint32_t p, const Sp
 }
 
 template <bool kPack>
-__device__ __forceinline__ void tile_fast(const SnapParams &P, const CrcTables &tb, char *chunk,
+__device__ __forceinline__ void tile_fast(const SnapParams &P, const char *ntab, const char *nf, char *chunk,
                                           const SegRow *rows, int nrows, uint32_t tile0, uint32_t *crc_out) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t lane4 = lane * 4;
     const uint32_t wbase = tile0 + warp * kWarpBytes + lane * kLaneSpan;
-    const char *nf = reinterpret_cast<const char *>(&tb.NF[0][0][0]);
     RowCursor rc;
     rc.init(rows, 0, nrows, wbase);
     auto load = [&](int r) -> Span {
@@ -280,25 +278,27 @@ __device__ __forceinline__ void tile_fast(const SnapParams &P, const CrcTables &
         if (r + kAhead < kRounds) buf[(r + kAhead) % (kAhead + 1)] = load(r + kAhead);
         Span &w = buf[r % (kAhead + 1)];
         if (kPack) st_span(chunk + wbase + r * kRound, w);
+#ifdef PCC_EXP_NOCRC  // timing experiment only: the copy without the CRC (wrong CRCs)
+        s ^= w.a.x ^ w.b.y;
+        continue;
+#endif
         uint4 w0 = w.a;
         w0.x ^= shift32(nf, lane4, s);  // the register, advanced over the gap, folded into w0
-        s = raw16(tb, lane4, w0);
+        s = raw16(ntab, lane4, w0);
         uint4 w1 = w.b;
         w1.x ^= s;
-        s = raw16(tb, lane4, w1);
+        s = raw16(ntab, lane4, w1);
         if (!kPack) scatter_span(rc, wbase + r * kRound, w);
     }
-    // lane -> end of this warp's 8 KiB (NL tables), XOR over the warp: the sub-tile's raw CRC
-    s = shift32(reinterpret_cast<const char *>(&tb.NL[0][0][0]), lane4, s);
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) s ^= __shfl_xor_sync(0xFFFFFFFFu, s, o);
-    if (lane == 0) crc_out[warp] = s;
+    // the lane's raw register, relative to the end of its last span (the finalize kernel
+    // shifts it to the warp-region end and XORs the warp's lanes)
+    crc_out[threadIdx.x] = s;
 }
 
 // Ragged tile (tile_len < kTile, a multiple of 16; only the last tile of a chunk): block-
 // strided words, generic shifts; the whole tile's CRC goes to the last sub-tile slot.
 template <bool kPack>
-__device__ __noinline__ void tile_generic(const SnapParams &P, const CrcTables &tb, char *chunk,
+__device__ __noinline__ void tile_generic(const SnapParams &P, const char *ntab, char *chunk,
                                           const SegRow *rows, int nrows, uint32_t tile0, uint32_t tile_len,
                                           uint32_t *crc_out, uint32_t *red) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -317,7 +317,7 @@ __device__ __noinline__ void tile_generic(const SnapParams &P, const CrcTables &
             scatter_word(rc, p, w);
         }
         if (any) s = multmodp(P.consts->x8n_stride, s);
-        s ^= raw16(tb, lane * 4, w);
+        s ^= raw16(ntab, lane * 4, w);
         e = p + 16;
         any = true;
     }
@@ -326,12 +326,12 @@ __device__ __noinline__ void tile_generic(const SnapParams &P, const CrcTables &
     for (int o = 16; o > 0; o >>= 1) c ^= __shfl_xor_sync(0xFFFFFFFFu, c, o);
     if (lane == 0) red[warp] = c;
     __syncthreads();
-    if (threadIdx.x < kWarps) {
-        uint32_t t = 0;
-        if (threadIdx.x == kWarps - 1)
-            for (int i = 0; i < kWarps; ++i) t ^= red[i];
-        crc_out[threadIdx.x] = t;  // slot kWarps-1 is relative to tile_end == chunk end
-    }
+    // the whole tile's raw CRC (relative to tile_end == chunk end) in the last lane of the last
+    // warp, whose lane shift is the identity; every other lane slot 0
+    uint32_t t = 0;
+    if (threadIdx.x == kThreads - 1)
+        for (int i = 0; i < kWarps; ++i) t ^= red[i];
+    crc_out[threadIdx.x] = t;
 }
 
 // The 96 KiB of tables arrive in shared memory by one TMA bulk copy (cp.async.bulk, completion
@@ -377,8 +377,9 @@ __device__ __forceinline__ void stage_rows(const SnapParams &P, uint2 tr, SegRow
 
 template <bool kPack>
 __global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
-    extern __shared__ __align__(128) uint8_t smem[];  // the 96 KiB of CRC tables
-    CrcTables &tb = *reinterpret_cast<CrcTables *>(smem);
+    extern __shared__ __align__(128) uint8_t smem[];  // NT + NF (kK1TableBytes)
+    const char *ntab = reinterpret_cast<const char *>(smem);
+    const char *nf = ntab + kNtBytes;
     __shared__ __align__(16) SegRow srows[2][kMaxTileRows];
     __shared__ uint32_t red[kWarps];
     __shared__ __align__(8) uint64_t tbar;
@@ -386,7 +387,7 @@ __global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
     const uint32_t G = gridDim.x;
     uint32_t item = blockIdx.x;
     uint2 tr = item_rows(P, item, n_items);
-    if (threadIdx.x == 0) tables_async_load(smem, P.tables, sizeof(CrcTables), &tbar);
+    if (threadIdx.x == 0) tables_async_load(smem, P.tables, kK1TableBytes, &tbar);
     stage_rows(P, tr, srows[0]);
     uint2 trn = item_rows(P, item + G, n_items);
     __syncthreads();  // mbarrier initialised before anyone waits on it
@@ -402,11 +403,11 @@ __global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
         char *chunk = P.ring_base + ((P.ring_head + j) % P.ring_slots) * P.chunk_bytes;
         const uint32_t tile0 = t * kTile;
         const uint64_t rem = P.chunk_bytes - tile0;
-        uint32_t *crc_out = P.tile_crc + ((uint64_t)j * P.tpc + t) * kWarps;
+        uint32_t *crc_out = P.tile_crc + ((uint64_t)j * P.tpc + t) * kWarps * kLaneOut;
         if (rem >= kTile)
-            tile_fast<kPack>(P, tb, chunk, rows, (int)tr.y, tile0, crc_out);
+            tile_fast<kPack>(P, ntab, nf, chunk, rows, (int)tr.y, tile0, crc_out);
         else
-            tile_generic<kPack>(P, tb, chunk, rows, (int)tr.y, tile0, (uint32_t)rem, crc_out, red);
+            tile_generic<kPack>(P, ntab, chunk, rows, (int)tr.y, tile0, (uint32_t)rem, crc_out, red);
         __syncthreads();  // srows[buf] and red[] are reused
         tr = trn;
         trn = trnn;
@@ -414,21 +415,44 @@ __global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
     cp_async_wait<0>();
 }
 
-// tiles -> chunk CRC (+ verify) -> slice digest.  One CTA per chunk.
-__global__ void __launch_bounds__(256) k_finalize(const FinalizeParams F) {
-    __shared__ uint32_t red[8];
+// lanes -> sub-tiles -> chunk CRC (+ verify) -> slice digest.  One CTA per chunk.  Each warp
+// takes 32 sub-tiles at a time: per sub-tile its 32 lane registers are shifted to the
+// sub-tile end (NL, one lane per thread: conflict-free) and XOR-reduced; lane k keeps
+// sub-tile k's value and then shifts it to the chunk end (multmodp, all lanes in parallel).
+constexpr int kFinThreads = 1024;
+__global__ void __launch_bounds__(kFinThreads) k_finalize(const FinalizeParams F) {
+    __shared__ __align__(16) uint32_t nl[kRegBytes / 4];
+    __shared__ uint32_t red[kFinThreads / 32];
+    for (uint32_t i = threadIdx.x; i < kRegBytes / 4; i += kFinThreads) nl[i] = F.tables->NL[i];
+    __syncthreads();
     const uint32_t j = blockIdx.x;
-    uint32_t v = 0;
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, lane4 = lane * 4;
     const uint32_t nsub = F.tpc * kWarps;
-    for (uint32_t t = threadIdx.x; t < nsub; t += blockDim.x)
-        v ^= multmodp(F.tile_shift[t], F.tile_crc[(uint64_t)j * nsub + t]);
+    const uint32_t *tc = F.tile_crc + (uint64_t)j * nsub * kLaneOut;
+    const char *nlt = reinterpret_cast<const char *>(nl);
+    uint32_t v = 0;
+    for (uint32_t base = warp * 32; base < nsub; base += kFinThreads) {
+        uint32_t mine = 0;
+        const uint32_t k_end = nsub - base < 32 ? nsub - base : 32;
+        uint32_t e[32];  // all 32 sub-tiles' lane values in flight at once
+#pragma unroll
+        for (uint32_t k = 0; k < 32; ++k) e[k] = k < k_end ? tc[(uint64_t)(base + k) * kLaneOut + lane] : 0u;
+#pragma unroll
+        for (uint32_t k = 0; k < 32; ++k) {
+            uint32_t x = shift32(nlt, lane4, e[k]);
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) x ^= __shfl_xor_sync(0xFFFFFFFFu, x, o);
+            if (lane == k) mine = x;
+        }
+        if (lane < k_end) v ^= multmodp(F.tile_shift[base + lane], mine);
+    }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v ^= __shfl_xor_sync(0xFFFFFFFFu, v, o);
-    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;
+    if (lane == 0) red[warp] = v;
     __syncthreads();
     if (threadIdx.x == 0) {
         uint32_t raw = 0;
-        for (int i = 0; i < (int)(blockDim.x >> 5); ++i) raw ^= red[i];
+        for (int i = 0; i < kFinThreads / 32; ++i) raw ^= red[i];
         const uint32_t crc = raw ^ F.ff[0] ^ 0xFFFFFFFFu;
         F.crc_out[j] = crc;
         if (F.expect) {
@@ -512,9 +536,9 @@ static int resident_ctas(int device) {
     if (device < 0 || device >= 64) return 1;
     if (!cached[device]) {
         int per_sm = 0, sms = 0;
-        cudaFuncSetAttribute(k_snapshot<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, sizeof(CrcTables));
-        cudaFuncSetAttribute(k_snapshot<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, sizeof(CrcTables));
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snapshot<true>, kThreads, sizeof(CrcTables));
+        cudaFuncSetAttribute(k_snapshot<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kK1TableBytes);
+        cudaFuncSetAttribute(k_snapshot<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kK1TableBytes);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snapshot<true>, kThreads, kK1TableBytes);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
         cached[device] = (per_sm > 0 ? per_sm : 1) * (sms > 0 ? sms : 1);
     }
@@ -530,19 +554,19 @@ int snapshot_grid(int device, uint32_t n_items, uint32_t cap) {
 
 cudaError_t launch_pack(const SnapParams &p, int grid, cudaStream_t s) {
     if (p.count == 0) return cudaSuccess;
-    k_snapshot<true><<<grid, kThreads, sizeof(CrcTables), s>>>(p);
+    k_snapshot<true><<<grid, kThreads, kK1TableBytes, s>>>(p);
     return cudaGetLastError();
 }
 
 cudaError_t launch_unpack(const SnapParams &p, int grid, cudaStream_t s) {
     if (p.count == 0) return cudaSuccess;
-    k_snapshot<false><<<grid, kThreads, sizeof(CrcTables), s>>>(p);
+    k_snapshot<false><<<grid, kThreads, kK1TableBytes, s>>>(p);
     return cudaGetLastError();
 }
 
 cudaError_t launch_finalize(const FinalizeParams &p, cudaStream_t s) {
     if (p.n == 0) return cudaSuccess;
-    k_finalize<<<p.n, 256, 0, s>>>(p);
+    k_finalize<<<p.n, kFinThreads, 0, s>>>(p);
     return cudaGetLastError();
 }
 

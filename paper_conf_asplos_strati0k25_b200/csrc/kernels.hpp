@@ -38,13 +38,14 @@ struct SnapParams {
     uint32_t first, count, tpc;
     char *ring_base;
     uint64_t ring_head, ring_slots;
-    uint32_t *tile_crc;          // [n * tpc * kWarps] raw sub-tile CRCs (relative to each sub-tile's end)
+    uint32_t *tile_crc;          // [n * tpc * kWarps * kLaneOut] raw lane CRCs (relative to each lane's last span end)
     const CrcTables *tables;
     const CrcConsts *consts;
 };
 
 struct FinalizeParams {
-    const uint32_t *tile_crc;
+    const uint32_t *tile_crc;    // K1/K2's lane CRCs, tile_crc_words(tpc) per chunk
+    const CrcTables *tables;     // NL (lane -> sub-tile end shifts)
     uint32_t n, tpc;             // sub-tiles per chunk = tpc * kWarps
     const uint32_t *tile_shift, *chunk_shift, *ff;
     uint32_t *crc_out;           // [n] standard CRC32C per chunk
@@ -52,6 +53,9 @@ struct FinalizeParams {
     uint32_t *bad;               // restore: [n] 1 = mismatch
     uint32_t *scratch;           // [4] zeroed: digest accumulator, done counter, n_bad, digest out
 };
+
+// words of K1/K2 lane-CRC output per chunk
+inline uint64_t tile_crc_words(uint32_t tpc) { return (uint64_t)tpc * kWarps * kLaneOut; }
 
 // Builds the CRC tables once per device (device memory owned by a process-wide cache).
 cudaError_t device_tables(int device, const CrcTables **tables, const CrcConsts **consts);

@@ -674,7 +674,7 @@ int pcc_register(pcc_ctx *c, const pcc_tensor *t, uint32_t nt) {
     const uint64_t nn = c->n ? c->n : 1;
     for (uint32_t s = 0; s < c->n_slots; ++s) {
         uint32_t *a = nullptr, *b = nullptr, *d = nullptr, *h = nullptr;
-        if ((e = cudaMalloc(&a, nn * c->geom.tpc * kWarps * sizeof(uint32_t))) != cudaSuccess)
+        if ((e = cudaMalloc(&a, nn * tile_crc_words(c->geom.tpc) * sizeof(uint32_t))) != cudaSuccess)
             return cuda_error(e, "tile crc");
         if ((e = cudaMalloc(&b, (nn + 1) * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "crc");
         if ((e = cudaMalloc(&d, 4 * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "scratch");
@@ -859,6 +859,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
     cudaMemsetAsync(c->scratch_dev[s], 0, 4 * sizeof(uint32_t), c->pack_stream);
     FinalizeParams F{};
     F.tile_crc = c->tile_crc_dev[s];
+    F.tables = c->tables;
     F.n = (uint32_t)c->n;
     F.tpc = c->geom.tpc;
     F.tile_shift = c->geom.tile_shift;
@@ -1181,6 +1182,7 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     PCC_TRACE("restore: copies + K2 issued t=%.0f us", c->now_us());
     FinalizeParams F{};
     F.tile_crc = tile;
+    F.tables = c->tables;
     F.n = (uint32_t)n;
     F.tpc = c->geom.tpc;
     F.tile_shift = c->geom.tile_shift;
@@ -1271,7 +1273,7 @@ int dp_fanout(pcc_ctx *c, uint32_t slot) {
     };
     // group size: bounded by 4 GiB of receive buffer
     uint64_t G = std::max<uint64_t>(1, std::min<uint64_t>(n_max, (4ull << 30) / (W * cb)));
-    const uint64_t nsub = (uint64_t)c->geom.tpc * kWarps;
+    const uint64_t nsub = tile_crc_words(c->geom.tpc);  // lane-CRC words per chunk
     if ((e = cudaMalloc(&rows, std::max<size_t>(1, full.rows.size()) * sizeof(SegRow))) ||
         (e = cudaMalloc(&rb, (C + 1) * 4)) || (e = cudaMalloc(&trows, std::max<size_t>(2, full.tile_rows.size()) * 4)) ||
         (e = cudaMalloc(&tile, C * nsub * 4)) || (e = cudaMalloc(&crc_mine, n_max * 4)) ||
@@ -1346,6 +1348,7 @@ int dp_fanout(pcc_ctx *c, uint32_t slot) {
             }
             FinalizeParams F{};
             F.tile_crc = tile + j0 * nsub;
+            F.tables = c->tables;
             F.n = (uint32_t)cnt;
             F.tpc = c->geom.tpc;
             F.tile_shift = g2.tile_shift;
