@@ -57,8 +57,8 @@ __host__ __device__ inline uint32_t x8n(const uint32_t *x2n, uint64_t n) {
 }
 
 // ---------------------------------------------------------------- kernel geometry
-// One CTA of 32 warps per SM (all warps share one copy of the tables), tile = 256 KiB of one
-// chunk, warp region = 8 KiB = 8 rounds of 1 KiB.  In round r lane l owns the 32 bytes at
+// One CTA of 32 warps per SM (all warps share one copy of the tables); the work item is an
+// 8 KiB tile of one chunk, owned by one warp = 8 rounds of 1 KiB.  In round r lane l owns the 32 bytes at
 // warp_base + r*1024 + 32*l: one 256-bit load and one 256-bit store per lane, so every warp
 // access is 1 KiB contiguous.  Loads run kAhead rounds ahead in registers.  Per round:
 //     x = shift(s, 992);  s = raw16(w0 ^ x);  s = raw16(w1 ^ s)
@@ -91,8 +91,7 @@ constexpr int kRounds = kWarpBytes / kRound;         // 8
 #endif
 constexpr int kAhead = PCC_KAHEAD;                   // rounds loaded ahead of the CRC (A/B builds: -DPCC_KAHEAD)
 constexpr uint32_t kGap = kRound - kLaneSpan;        // zero bytes between a lane's spans
-constexpr uint32_t kTile = kWarps * kWarpBytes;      // 256 KiB per CTA tile
-constexpr int kMaxTileRows = 512;                    // segment rows staged per tile (more -> read from global)
+constexpr uint32_t kTile = kWarpBytes;               // a work item: one warp's 8 KiB of one chunk
 constexpr int kLaneOut = 32;                         // raw CRCs K1/K2 write per warp sub-tile (one per lane)
 
 #ifndef PCC_NTBITS
@@ -117,13 +116,13 @@ struct CrcTables {
 };
 constexpr uint32_t kK1TableBytes = kNtBytes + kRegBytes;
 static_assert(kK1TableBytes % 16 == 0, "TMA bulk copy size");
-static_assert(kK1TableBytes + 2 * kMaxTileRows * 16 + 1024 <= 227 * 1024, "K1 shared memory");
+static_assert(kK1TableBytes + 1024 <= 227 * 1024, "K1 shared memory");
 
 // Constants that do not need a table.
 struct CrcConsts {
     uint32_t x2n[kX2n];
     uint32_t warp_shift[kWarps];  // x8n((kWarps-1-w) * kWarpBytes)
-    uint32_t x8n_stride;          // x8n(kThreads*16): generic (ragged-tile) path, one thread stride
+    uint32_t x8n_stride;          // x8n(32*16): generic (ragged-tile) path, one warp stride
 };
 
 // x >> k as IMAD.HI on the FMA pipe (a plain >> becomes SHF on the ALU pipe, which the

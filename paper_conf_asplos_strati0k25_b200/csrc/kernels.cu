@@ -79,14 +79,14 @@ __global__ void k_build_tables(CrcTables *tb, CrcConsts *cs) {
     }
     if (t < kX2n) cs->x2n[t] = x2n[t];
     if (t < kWarps) cs->warp_shift[t] = x8n(x2n, (uint64_t)(kWarps - 1 - t) * kWarpBytes);
-    if (t == 0) cs->x8n_stride = x8n(x2n, (uint64_t)kThreads * 16);
+    if (t == 0) cs->x8n_stride = x8n(x2n, 32 * 16);
 }
 
 __global__ void k_setup_geometry(uint32_t *tile_shift, uint32_t *chunk_shift, uint32_t *ff, const CrcConsts *cs,
                                  uint64_t cb, uint32_t n, uint32_t tpc) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
-    if (i < tpc * kWarps) {  // sub-tile (t, w) = warp w's 8 KiB of tile t
-        uint64_t end = (uint64_t)(i / kWarps) * kTile + (uint64_t)(i % kWarps + 1) * kWarpBytes;
+    if (i < tpc) {  // tile i = one warp's 8 KiB
+        uint64_t end = (uint64_t)(i + 1) * kTile;
         if (end > cb) end = cb;
         tile_shift[i] = x8n(cs->x2n, cb - end);
     }
@@ -110,11 +110,21 @@ __device__ __forceinline__ void st_stream(void *p, uint4 v) {
                  : "memory");
 }
 
+// one 16-byte segment row through the read-only (L1-cached) path
+__device__ __forceinline__ SegRow ld_row(const SegRow *p) {
+    const uint4 v = __ldg(reinterpret_cast<const uint4 *>(p));
+    SegRow r;
+    r.ptr = ((uint64_t)v.y << 32) | v.x;
+    r.dst_off = v.z;
+    r.len = v.w;
+    return r;
+}
+
 // first row in [lo, hi) whose end (dst_off + len) is > pos
 __device__ __forceinline__ int lower_row(const SegRow *rows, int lo, int hi, uint32_t pos) {
     while (lo < hi) {
         int mid = (lo + hi) >> 1;
-        SegRow r = rows[mid];
+        const SegRow r = ld_row(rows + mid);
         if (r.dst_off + r.len <= pos) lo = mid + 1; else hi = mid;
     }
     return lo;
@@ -134,7 +144,7 @@ struct RowCursor {
     }
     __device__ __forceinline__ void load() {
         if (cur < end) {
-            SegRow r = rows[cur];
+            const SegRow r = ld_row(rows + cur);
             ptr = r.ptr;
             off = r.dst_off;
             stop = r.dst_off + r.len;
@@ -219,16 +229,22 @@ struct Span {  // one lane's 32 bytes of a round
     uint4 a, b;
 };
 
+#ifndef PCC_EXP_LD
+#define PCC_EXP_LD "ld.global.nc.L1::no_allocate.v8.u32"
+#endif
+#ifndef PCC_EXP_ST
+#define PCC_EXP_ST "st.global.cs.v8.u32"
+#endif
 __device__ __forceinline__ Span ld_span(const void *p) {  // 256-bit streaming load
     Span v;
-    asm volatile("ld.global.nc.L1::no_allocate.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+    asm volatile(PCC_EXP_LD " {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
                  : "=r"(v.a.x), "=r"(v.a.y), "=r"(v.a.z), "=r"(v.a.w), "=r"(v.b.x), "=r"(v.b.y), "=r"(v.b.z),
                    "=r"(v.b.w)
                  : "l"(p));
     return v;
 }
 __device__ __forceinline__ void st_span(void *p, const Span &v) {  // 256-bit streaming store
-    asm volatile("st.global.cs.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(v.a.x), "r"(v.a.y),
+    asm volatile(PCC_EXP_ST " [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(v.a.x), "r"(v.a.y),
                  "r"(v.a.z), "r"(v.a.w), "r"(v.b.x), "r"(v.b.y), "r"(v.b.z), "r"(v.b.w)
                  : "memory");
 }
@@ -258,12 +274,12 @@ __device__ __forceinline__ void scatter_span(RowCursor &rc, uint32_t p, const Sp
     scatter_word(rc, p + 16, v.b);
 }
 
+// One warp, one 8 KiB tile: 8 rounds of 1 KiB, lane l moves the 32 bytes at 32*l of each round.
 template <bool kPack>
-__device__ __forceinline__ void tile_fast(const SnapParams &P, const char *ntab, const char *nf, char *chunk,
-                                          const SegRow *rows, int nrows, uint32_t tile0, uint32_t *crc_out) {
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+__device__ __forceinline__ void tile_fast(const char *ntab, const char *nf, char *chunk, const SegRow *rows, int nrows,
+                                          uint32_t tile0, uint32_t lane, uint32_t *crc_out) {
     const uint32_t lane4 = lane * 4;
-    const uint32_t wbase = tile0 + warp * kWarpBytes + lane * kLaneSpan;
+    const uint32_t wbase = tile0 + lane * kLaneSpan;
     RowCursor rc;
     rc.init(rows, 0, nrows, wbase);
     auto load = [&](int r) -> Span {
@@ -291,23 +307,23 @@ __device__ __forceinline__ void tile_fast(const SnapParams &P, const char *ntab,
         if (!kPack) scatter_span(rc, wbase + r * kRound, w);
     }
     // the lane's raw register, relative to the end of its last span (the finalize kernel
-    // shifts it to the warp-region end and XORs the warp's lanes)
-    crc_out[threadIdx.x] = s;
+    // shifts it to the tile end and XORs the warp's lanes)
+    crc_out[lane] = s;
 }
 
-// Ragged tile (tile_len < kTile, a multiple of 16; only the last tile of a chunk): block-
-// strided words, generic shifts; the whole tile's CRC goes to the last sub-tile slot.
+// Ragged tile (tile_len < kTile, a multiple of 16; only the last tile of a chunk): warp-
+// strided 16-byte words, generic shifts; the whole tile's raw CRC (relative to tile_end ==
+// chunk end) goes to lane 31's slot, whose lane shift is the identity; the other slots get 0.
 template <bool kPack>
-__device__ __noinline__ void tile_generic(const SnapParams &P, const char *ntab, char *chunk,
-                                          const SegRow *rows, int nrows, uint32_t tile0, uint32_t tile_len,
-                                          uint32_t *crc_out, uint32_t *red) {
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+__device__ __noinline__ void tile_generic(const SnapParams &P, const char *ntab, char *chunk, const SegRow *rows,
+                                          int nrows, uint32_t tile0, uint32_t tile_len, uint32_t lane,
+                                          uint32_t *crc_out) {
     const uint32_t tile_end = tile0 + tile_len;
     RowCursor rc;
-    rc.init(rows, 0, nrows, tile0 + threadIdx.x * 16);
+    rc.init(rows, 0, nrows, tile0 + lane * 16);
     uint32_t s = 0, e = 0;
     bool any = false;
-    for (uint32_t p = tile0 + threadIdx.x * 16; p < tile_end; p += kThreads * 16) {
+    for (uint32_t p = tile0 + lane * 16; p < tile_end; p += 32 * 16) {
         uint4 w;
         if (kPack) {
             w = gather_word(rc, p);
@@ -324,18 +340,11 @@ __device__ __noinline__ void tile_generic(const SnapParams &P, const char *ntab,
     uint32_t c = any ? multmodp(x8n(P.consts->x2n, tile_end - e), s) : 0u;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) c ^= __shfl_xor_sync(0xFFFFFFFFu, c, o);
-    if (lane == 0) red[warp] = c;
-    __syncthreads();
-    // the whole tile's raw CRC (relative to tile_end == chunk end) in the last lane of the last
-    // warp, whose lane shift is the identity; every other lane slot 0
-    uint32_t t = 0;
-    if (threadIdx.x == kThreads - 1)
-        for (int i = 0; i < kWarps; ++i) t ^= red[i];
-    crc_out[threadIdx.x] = t;
+    crc_out[lane] = lane == 31 ? c : 0u;
 }
 
-// The 96 KiB of tables arrive in shared memory by one TMA bulk copy (cp.async.bulk, completion
-// on an mbarrier) while the first tile's rows are being staged.
+// The tables arrive in shared memory by one TMA bulk copy (cp.async.bulk, completion on an
+// mbarrier) while the warps fetch their first tiles' row descriptors.
 __device__ __forceinline__ void tables_async_load(void *smem, const void *gmem, uint32_t bytes, uint64_t *bar) {
     const uint32_t sbar = (uint32_t)__cvta_generic_to_shared(bar);
     const uint32_t sdst = (uint32_t)__cvta_generic_to_shared(smem);
@@ -362,57 +371,45 @@ __device__ __forceinline__ void tables_wait(uint64_t *bar) {
 __device__ __forceinline__ uint2 item_rows(const SnapParams &P, uint32_t item, uint32_t n_items) {
     if (item >= n_items) return make_uint2(0, 0);
     const uint32_t jl = item / P.tpc, t = item - jl * P.tpc;
-    return P.tile_rows[(uint64_t)(P.first + jl) * P.tpc + t];
+    return __ldg(P.tile_rows + (uint64_t)(P.first + jl) * P.tpc + t);
 }
 
-// cp.async (LDGSTS) of a tile's segment rows into one of two shared buffers; one commit group
-__device__ __forceinline__ void stage_rows(const SnapParams &P, uint2 tr, SegRow *dst) {
-    const uint32_t k = tr.y <= (uint32_t)kMaxTileRows ? tr.y : 0u;
-    for (uint32_t i = threadIdx.x; i < k; i += kThreads) {
-        const uint32_t sd = (uint32_t)__cvta_generic_to_shared(dst + i);
-        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sd), "l"(P.rows + tr.x + i) : "memory");
-    }
-    asm volatile("cp.async.commit_group;" ::: "memory");
-}
-
+// K1 (kPack) / K2.  Work item = one 8 KiB tile of one chunk, owned by one warp; warps stride
+// over the items independently (no block barrier after the table load), each fetching its
+// next tile's row descriptor one tile ahead.
 template <bool kPack>
 __global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
     extern __shared__ __align__(128) uint8_t smem[];  // NT + NF (kK1TableBytes)
     const char *ntab = reinterpret_cast<const char *>(smem);
     const char *nf = ntab + kNtBytes;
-    __shared__ __align__(16) SegRow srows[2][kMaxTileRows];
-    __shared__ uint32_t red[kWarps];
     __shared__ __align__(8) uint64_t tbar;
+    const uint32_t lane = threadIdx.x & 31;
     const uint32_t n_items = P.count * P.tpc;
-    const uint32_t G = gridDim.x;
-    uint32_t item = blockIdx.x;
-    uint2 tr = item_rows(P, item, n_items);
+    const uint32_t stride = gridDim.x * kWarps;
+    uint32_t item = blockIdx.x * kWarps + (threadIdx.x >> 5);
+    // 256-bit accesses need 32-B aligned chunks (chunk_bytes is only required to be a multiple
+    // of 16; the ring / slot bases are 256-B aligned)
+    const bool fast_ok = (P.chunk_bytes % 32) == 0 && (reinterpret_cast<uintptr_t>(P.ring_base) % 32) == 0;
     if (threadIdx.x == 0) tables_async_load(smem, P.tables, kK1TableBytes, &tbar);
-    stage_rows(P, tr, srows[0]);
-    uint2 trn = item_rows(P, item + G, n_items);
+    uint2 tr = item_rows(P, item, n_items);
     __syncthreads();  // mbarrier initialised before anyone waits on it
     tables_wait(&tbar);
-    for (int buf = 0; item < n_items; item += G, buf ^= 1) {
-        cp_async_wait<0>();  // this tile's rows (the only group in flight here)
-        __syncthreads();
-        stage_rows(P, trn, srows[buf ^ 1]);  // the next tile's rows, in flight during this one
-        const uint2 trnn = item_rows(P, item + 2 * G, n_items);
-        const SegRow *rows = tr.y <= (uint32_t)kMaxTileRows ? srows[buf] : P.rows + tr.x;
+    for (; item < n_items; item += stride) {
+        const uint2 trn = item_rows(P, item + stride, n_items);
         const uint32_t jl = item / P.tpc, t = item - jl * P.tpc;
         const uint32_t j = P.first + jl;
         char *chunk = P.ring_base + ((P.ring_head + j) % P.ring_slots) * P.chunk_bytes;
         const uint32_t tile0 = t * kTile;
         const uint64_t rem = P.chunk_bytes - tile0;
-        uint32_t *crc_out = P.tile_crc + ((uint64_t)j * P.tpc + t) * kWarps * kLaneOut;
-        if (rem >= kTile)
-            tile_fast<kPack>(P, ntab, nf, chunk, rows, (int)tr.y, tile0, crc_out);
+        uint32_t *crc_out = P.tile_crc + ((uint64_t)j * P.tpc + t) * kLaneOut;
+        const SegRow *rows = P.rows + tr.x;
+        if (rem >= kTile && fast_ok)
+            tile_fast<kPack>(ntab, nf, chunk, rows, (int)tr.y, tile0, lane, crc_out);
         else
-            tile_generic<kPack>(P, ntab, chunk, rows, (int)tr.y, tile0, (uint32_t)rem, crc_out, red);
-        __syncthreads();  // srows[buf] and red[] are reused
+            tile_generic<kPack>(P, ntab, chunk, rows, (int)tr.y, tile0, rem < kTile ? (uint32_t)rem : kTile, lane,
+                                crc_out);
         tr = trn;
-        trn = trnn;
     }
-    cp_async_wait<0>();
 }
 
 // lanes -> sub-tiles -> chunk CRC (+ verify) -> slice digest.  One CTA per chunk.  Each warp
@@ -427,7 +424,7 @@ __global__ void __launch_bounds__(kFinThreads) k_finalize(const FinalizeParams F
     __syncthreads();
     const uint32_t j = blockIdx.x;
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, lane4 = lane * 4;
-    const uint32_t nsub = F.tpc * kWarps;
+    const uint32_t nsub = F.tpc;  // tiles per chunk, 32 lane values each
     const uint32_t *tc = F.tile_crc + (uint64_t)j * nsub * kLaneOut;
     const char *nlt = reinterpret_cast<const char *>(nl);
     uint32_t v = 0;
@@ -516,10 +513,10 @@ cudaError_t setup_geometry(DevGeometry *g, uint64_t chunk_bytes, uint32_t n, cud
     g->chunk_bytes = chunk_bytes;
     g->n = n;
     g->tpc = (uint32_t)((chunk_bytes + kTile - 1) / kTile);
-    if ((e = cudaMalloc(&g->tile_shift, sizeof(uint32_t) * g->tpc * kWarps)) != cudaSuccess) return e;
+    if ((e = cudaMalloc(&g->tile_shift, sizeof(uint32_t) * g->tpc)) != cudaSuccess) return e;
     if ((e = cudaMalloc(&g->chunk_shift, sizeof(uint32_t) * (n ? n : 1))) != cudaSuccess) return e;
     if ((e = cudaMalloc(&g->ff, sizeof(uint32_t) * 2)) != cudaSuccess) return e;
-    const uint32_t m = g->tpc * kWarps > n ? g->tpc * kWarps : (n ? n : 1);
+    const uint32_t m = g->tpc > n ? g->tpc : (n ? n : 1);
     k_setup_geometry<<<(m + 255) / 256, 256, 0, s>>>(g->tile_shift, g->chunk_shift, g->ff, cs, chunk_bytes, n, g->tpc);
     return cudaGetLastError();
 }
@@ -545,10 +542,11 @@ static int resident_ctas(int device) {
     return cached[device];
 }
 
-int snapshot_grid(int device, uint32_t n_items, uint32_t cap) {
+int snapshot_grid(int device, uint32_t n_items, uint32_t cap) {  // n_items = 8 KiB tiles (one warp each)
     int g = resident_ctas(device);
     if (cap && (int)cap < g) g = (int)cap;
-    if ((uint32_t)g > n_items) g = (int)n_items;
+    const uint32_t need = (n_items + kWarps - 1) / kWarps;
+    if ((uint32_t)g > need) g = (int)need;
     return g < 1 ? 1 : g;
 }
 

@@ -21,8 +21,8 @@ static_assert(sizeof(SegRow) == 16, "SegRow");
 struct DevGeometry {
     uint64_t chunk_bytes = 0;
     uint32_t n = 0;              // chunks in this rank's slice
-    uint32_t tpc = 0;            // tiles per chunk = ceil(chunk_bytes / kTile)
-    uint32_t *tile_shift = nullptr;   // [tpc*kWarps] x8n(CB - end of sub-tile (t, w)) (a sub-tile = one warp's 8 KiB)
+    uint32_t tpc = 0;            // tiles per chunk = ceil(chunk_bytes / kTile), a tile = one warp's 8 KiB
+    uint32_t *tile_shift = nullptr;   // [tpc] x8n(CB - end of tile t)
     uint32_t *chunk_shift = nullptr;  // [n]    x8n((n-1-j) * CB)
     uint32_t *ff = nullptr;           // [2]    shift(~0, CB), shift(~0, n*CB)
 };
@@ -38,7 +38,7 @@ struct SnapParams {
     uint32_t first, count, tpc;
     char *ring_base;
     uint64_t ring_head, ring_slots;
-    uint32_t *tile_crc;          // [n * tpc * kWarps * kLaneOut] raw lane CRCs (relative to each lane's last span end)
+    uint32_t *tile_crc;          // [n * tpc * kLaneOut] raw lane CRCs (relative to each lane's last span end)
     const CrcTables *tables;
     const CrcConsts *consts;
 };
@@ -46,7 +46,7 @@ struct SnapParams {
 struct FinalizeParams {
     const uint32_t *tile_crc;    // K1/K2's lane CRCs, tile_crc_words(tpc) per chunk
     const CrcTables *tables;     // NL (lane -> sub-tile end shifts)
-    uint32_t n, tpc;             // sub-tiles per chunk = tpc * kWarps
+    uint32_t n, tpc;             // tiles per chunk
     const uint32_t *tile_shift, *chunk_shift, *ff;
     uint32_t *crc_out;           // [n] standard CRC32C per chunk
     const uint32_t *expect;      // restore: [n] expected CRCs (nullptr when packing)
@@ -55,7 +55,7 @@ struct FinalizeParams {
 };
 
 // words of K1/K2 lane-CRC output per chunk
-inline uint64_t tile_crc_words(uint32_t tpc) { return (uint64_t)tpc * kWarps * kLaneOut; }
+inline uint64_t tile_crc_words(uint32_t tpc) { return (uint64_t)tpc * kLaneOut; }
 
 // Builds the CRC tables once per device (device memory owned by a process-wide cache).
 cudaError_t device_tables(int device, const CrcTables **tables, const CrcConsts **consts);
