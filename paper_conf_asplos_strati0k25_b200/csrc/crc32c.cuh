@@ -90,7 +90,16 @@ constexpr int kRounds = kWarpBytes / kRound;         // 8
 #define PCC_KAHEAD 1
 #endif
 constexpr int kAhead = PCC_KAHEAD;                   // rounds loaded ahead of the CRC (A/B builds: -DPCC_KAHEAD)
-constexpr uint32_t kGap = kRound - kLaneSpan;        // zero bytes between a lane's spans
+#ifndef PCC_KRUN
+#define PCC_KRUN 1
+#endif
+// A lane's spans are contiguous for kRun rounds (a "run" of kRun*32 B); round r of lane l sits
+// at (r / kRun) * kRun*kRound + l * kRun*kLaneSpan + (r % kRun) * kLaneSpan of the warp tile.
+// kRun = 1: every warp access is 1 KiB contiguous and the register crosses a gap every round;
+// larger kRun trades coalescing for fewer gap shifts (none at kRun = kRounds).
+constexpr int kRun = PCC_KRUN;                       // (A/B builds: -DPCC_KRUN)
+constexpr uint32_t kLaneRun = kRun * kLaneSpan;      // contiguous bytes of one lane
+constexpr uint32_t kGap = kRun * kRound - kLaneRun;  // zero bytes between a lane's runs
 constexpr uint32_t kTile = kWarpBytes;               // a work item: one warp's 8 KiB of one chunk
 constexpr int kLaneOut = 32;                         // raw CRCs K1/K2 write per warp sub-tile (one per lane)
 
@@ -112,7 +121,7 @@ constexpr uint32_t kRegBytes = (kG32 - 1) * kRegTab + (1u << 2) * 128;
 struct CrcTables {
     uint32_t NT[kNtBytes / 4];   // NT[t][v][l] = raw16(16-byte word whose bits [kNtBits*t, +kNtBits) are v)
     uint32_t NF[kRegBytes / 4];  // NF[g][v][l] = shift(v << 5g, kGap): the zeros before a lane's next span
-    uint32_t NL[kRegBytes / 4];  // NL[g][v][l] = shift(v << 5g, kLaneSpan*(31-l)): lane -> warp-region end
+    uint32_t NL[kRegBytes / 4];  // NL[g][v][l] = shift(v << 5g, kLaneRun*(31-l)): lane -> warp-region end
 };
 constexpr uint32_t kK1TableBytes = kNtBytes + kRegBytes;
 static_assert(kK1TableBytes % 16 == 0, "TMA bulk copy size");

@@ -9,16 +9,18 @@
 // moved verbatim, so NaN payloads / denormals survive (R1).
 //
 // Execution model:
-//   * one CTA of 32 warps per SM (the tables fill its shared memory), tile = 256 KiB of one
-//     chunk, grid-stride over (chunk, tile) items; grid = SMs (or the pack_ctas cap);
-//   * a warp owns 8 KiB of the tile = 8 rounds of 1 KiB: lane l moves the 32 bytes at
-//     32*l with one 256-bit load and one 256-bit store, one round of loads ahead;
+//   * one CTA of 32 warps per SM (the tables fill its shared memory); the work item is an
+//     8 KiB tile of one chunk, owned by one warp; warps stride over the items independently
+//     (no block barrier after the TMA table load); grid = SMs (or the pack_ctas cap);
+//   * a tile is 8 rounds of 1 KiB: lane l moves the 32 bytes at 32*l with one 256-bit load and
+//     one 256-bit store, one round of loads ahead;
 //   * the segment-table row under each word is tracked by a per-lane cursor over the tile's
-//     rows (staged in shared memory by cp.async); a 16-B word holds bytes of at most one row
-//     because rows start 16-B aligned in the chunk;
+//     rows (read through L1; descriptors fetched items ahead); a 16-B word holds bytes of at
+//     most one row because rows start 16-B aligned in the chunk;
 //   * CRC (crc32c.cuh): per-lane register, advanced over the gap by the NF tables and fed the
 //     words through the 6-bit NT tables (51 conflict-free LDS per 32 B); every lane writes its
-//     register, and k_finalize folds lanes -> 8 KiB sub-tiles -> chunks -> slice digest.
+//     register; k_fold_subtiles folds lanes -> 8 KiB sub-tiles -> shares of chunks on the whole
+//     GPU and k_chunk_crcs chunk shares -> chunk CRCs -> slice digest.
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <mutex>
@@ -74,8 +76,8 @@ __global__ void k_build_tables(CrcTables *tb, CrcConsts *cs) {
     for (uint32_t e = t; e < kRegBytes / 4; e += blockDim.x) {
         const uint32_t g = e >> 10, v = (e >> 5) & 31, l = e & 31;
         tb->NF[e] = vf[g][v];
-        // NL: lane-specific shift kLaneSpan*(31-l)
-        tb->NL[e] = multmodp(x8n(x2n, kLaneSpan * (31 - l)), (uint32_t)((uint64_t)v << (5 * g)));
+        // NL: lane-specific shift kLaneRun*(31-l)
+        tb->NL[e] = multmodp(x8n(x2n, kLaneRun * (31 - l)), (uint32_t)((uint64_t)v << (5 * g)));
     }
     if (t < kX2n) cs->x2n[t] = x2n[t];
     if (t < kWarps) cs->warp_shift[t] = x8n(x2n, (uint64_t)(kWarps - 1 - t) * kWarpBytes);
@@ -279,12 +281,12 @@ template <bool kPack>
 __device__ __forceinline__ void tile_fast(const char *ntab, const char *nf, char *chunk, const SegRow *rows, int nrows,
                                           uint32_t tile0, uint32_t lane, uint32_t *crc_out) {
     const uint32_t lane4 = lane * 4;
-    const uint32_t wbase = tile0 + lane * kLaneSpan;
+    const uint32_t wbase = tile0 + lane * kLaneRun;
+    // chunk position of round r (compile-time offset once unrolled)
+    auto pos = [&](int r) -> uint32_t { return wbase + (r / kRun) * (kRun * kRound) + (r % kRun) * kLaneSpan; };
     RowCursor rc;
     rc.init(rows, 0, nrows, wbase);
-    auto load = [&](int r) -> Span {
-        return kPack ? gather_span(rc, wbase + r * kRound) : ld_span(chunk + wbase + r * kRound);
-    };
+    auto load = [&](int r) -> Span { return kPack ? gather_span(rc, pos(r)) : ld_span(chunk + pos(r)); };
     Span buf[kAhead + 1];
 #pragma unroll
     for (int r = 0; r < kAhead; ++r) buf[r] = load(r);
@@ -293,18 +295,20 @@ __device__ __forceinline__ void tile_fast(const char *ntab, const char *nf, char
     for (int r = 0; r < kRounds; ++r) {
         if (r + kAhead < kRounds) buf[(r + kAhead) % (kAhead + 1)] = load(r + kAhead);
         Span &w = buf[r % (kAhead + 1)];
-        if (kPack) st_span(chunk + wbase + r * kRound, w);
+        if (kPack) st_span(chunk + pos(r), w);
 #ifdef PCC_EXP_NOCRC  // timing experiment only: the copy without the CRC (wrong CRCs)
         s ^= w.a.x ^ w.b.y;
         continue;
 #endif
         uint4 w0 = w.a;
-        w0.x ^= shift32(nf, lane4, s);  // the register, advanced over the gap, folded into w0
+        // the register folded into w0; advanced over the gap first when a new run starts
+        // (never in round 0, where it is still 0)
+        w0.x ^= (r > 0 && r % kRun == 0) ? shift32(nf, lane4, s) : s;
         s = raw16(ntab, lane4, w0);
         uint4 w1 = w.b;
         w1.x ^= s;
         s = raw16(ntab, lane4, w1);
-        if (!kPack) scatter_span(rc, wbase + r * kRound, w);
+        if (!kPack) scatter_span(rc, pos(r), w);
     }
     // the lane's raw register, relative to the end of its last span (the finalize kernel
     // shifts it to the tile end and XORs the warp's lanes)
@@ -374,6 +378,39 @@ __device__ __forceinline__ uint2 item_rows(const SnapParams &P, uint32_t item, u
     return __ldg(P.tile_rows + (uint64_t)(P.first + jl) * P.tpc + t);
 }
 
+__device__ __forceinline__ void prefetch_l2_bulk(uint64_t addr, uint32_t bytes) {  // addr, bytes: 16-B multiples
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(addr), "r"(bytes) : "memory");
+}
+
+// Warm L2 with the bytes of the warp's NEXT work item while it works on this one (a TMA bulk
+// prefetch per segment row; rounded inwards to 16 B, so it never touches bytes outside a row):
+// the item's loads then hit L2 instead of waiting out HBM latency with one round in registers.
+template <bool kPack>
+__device__ __forceinline__ void prefetch_item(const SnapParams &P, uint32_t item, uint32_t n_items, uint2 tr,
+                                              uint32_t lane) {
+    if (item >= n_items) return;
+    const uint32_t jl = item / P.tpc, t = item - jl * P.tpc;
+    const uint64_t tile0 = (uint64_t)t * kTile;
+    const uint64_t tile_end = tile0 + kTile < P.chunk_bytes ? tile0 + kTile : P.chunk_bytes;
+    if (!kPack) {  // K2 reads the staged chunk: one contiguous range
+        if (lane == 0) {
+            const char *chunk = P.ring_base + ((P.ring_head + P.first + jl) % P.ring_slots) * P.chunk_bytes;
+            prefetch_l2_bulk(reinterpret_cast<uint64_t>(chunk + tile0), (uint32_t)(tile_end - tile0) & ~15u);
+        }
+        return;
+    }
+    for (uint32_t i = lane; i < tr.y; i += 32) {
+        const SegRow r = ld_row(P.rows + tr.x + i);
+        const uint64_t lo = r.dst_off > tile0 ? r.dst_off : tile0;
+        const uint64_t re = (uint64_t)r.dst_off + r.len;
+        const uint64_t hi = re < tile_end ? re : tile_end;
+        if (hi <= lo) continue;
+        const uint64_t src = r.ptr + (lo - r.dst_off);
+        const uint64_t a = (src + 15) & ~15ull, b = (src + (hi - lo)) & ~15ull;
+        if (b > a) prefetch_l2_bulk(a, (uint32_t)(b - a));
+    }
+}
+
 // K1 (kPack) / K2.  Work item = one 8 KiB tile of one chunk, owned by one warp; warps stride
 // over the items independently (no block barrier after the table load), each fetching its
 // next tile's row descriptor one tile ahead.
@@ -392,10 +429,15 @@ __global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
     const bool fast_ok = (P.chunk_bytes % 32) == 0 && (reinterpret_cast<uintptr_t>(P.ring_base) % 32) == 0;
     if (threadIdx.x == 0) tables_async_load(smem, P.tables, kK1TableBytes, &tbar);
     uint2 tr = item_rows(P, item, n_items);
+    uint2 trn = item_rows(P, item + stride, n_items);
     __syncthreads();  // mbarrier initialised before anyone waits on it
+#ifdef PCC_L2PF
+    prefetch_item<kPack>(P, item + stride, n_items, trn, lane);
+#endif
     tables_wait(&tbar);
     for (; item < n_items; item += stride) {
-        const uint2 trn = item_rows(P, item + stride, n_items);
+        // descriptors two items ahead; the next item's bytes are warmed in L2 one item ahead
+        const uint2 trnn = item_rows(P, item + 2 * stride, n_items);
         const uint32_t jl = item / P.tpc, t = item - jl * P.tpc;
         const uint32_t j = P.first + jl;
         char *chunk = P.ring_base + ((P.ring_head + j) % P.ring_slots) * P.chunk_bytes;
@@ -409,61 +451,110 @@ __global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
             tile_generic<kPack>(P, ntab, chunk, rows, (int)tr.y, tile0, rem < kTile ? (uint32_t)rem : kTile, lane,
                                 crc_out);
         tr = trn;
+        trn = trnn;
+#ifdef PCC_L2PF
+        prefetch_item<kPack>(P, item + 2 * stride, n_items, trn, lane);
+#endif
     }
 }
 
-// lanes -> sub-tiles -> chunk CRC (+ verify) -> slice digest.  One CTA per chunk.  Each warp
-// takes 32 sub-tiles at a time: per sub-tile its 32 lane registers are shifted to the
-// sub-tile end (NL, one lane per thread: conflict-free) and XOR-reduced; lane k keeps
-// sub-tile k's value and then shifts it to the chunk end (multmodp, all lanes in parallel).
-constexpr int kFinThreads = 1024;
-__global__ void __launch_bounds__(kFinThreads) k_finalize(const FinalizeParams F) {
+// lanes -> sub-tiles -> chunk CRC (+ verify) -> slice digest, in two kernels so that the whole
+// GPU shares the work (one CTA per chunk left most SMs idle: 33 us for the 66 chunks of C2).
+//
+// k_fold_subtiles: persistent CTAs (one per SM) load the lane-shift tables NL into shared
+// memory once, then take work units (j, s) = chunk j's sub-tiles [s*kFoldSub, +kFoldSub); each
+// warp 32 of them: per sub-tile its 32 lane registers are shifted to the sub-tile end (NL, one
+// lane per bank: conflict-free) and XOR-reduced; lane k keeps sub-tile k's value and shifts it
+// to the chunk end (multmodp, all lanes in parallel).  The unit's XOR is the raw CRC of its
+// share of the chunk relative to the chunk end; it is written over the first word of the
+// unit's own lane-CRC region (read only by this unit, and consumed before the write).
+constexpr int kFoldThreads = 1024;
+constexpr uint32_t kFoldSub = kFoldThreads;  // sub-tiles per work unit: 32 per warp
+__host__ __device__ inline uint32_t fold_splits(uint32_t tpc) { return (tpc + kFoldSub - 1) / kFoldSub; }
+
+__global__ void __launch_bounds__(kFoldThreads) k_fold_subtiles(const FinalizeParams F) {
     __shared__ __align__(16) uint32_t nl[kRegBytes / 4];
-    __shared__ uint32_t red[kFinThreads / 32];
-    for (uint32_t i = threadIdx.x; i < kRegBytes / 4; i += kFinThreads) nl[i] = F.tables->NL[i];
+    __shared__ uint32_t red[kFoldThreads / 32];
+    for (uint32_t i = threadIdx.x; i < kRegBytes / 4; i += kFoldThreads) nl[i] = F.tables->NL[i];
     __syncthreads();
-    const uint32_t j = blockIdx.x;
+    const uint32_t S = fold_splits(F.tpc);
     const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31, lane4 = lane * 4;
     const uint32_t nsub = F.tpc;  // tiles per chunk, 32 lane values each
-    const uint32_t *tc = F.tile_crc + (uint64_t)j * nsub * kLaneOut;
     const char *nlt = reinterpret_cast<const char *>(nl);
-    uint32_t v = 0;
-    for (uint32_t base = warp * 32; base < nsub; base += kFinThreads) {
-        uint32_t mine = 0;
-        const uint32_t k_end = nsub - base < 32 ? nsub - base : 32;
-        uint32_t e[32];  // all 32 sub-tiles' lane values in flight at once
+    for (uint32_t u = blockIdx.x; u < F.n * S; u += gridDim.x) {
+        const uint32_t j = u / S, s = u - j * S;
+        uint32_t *tc = F.tile_crc + (uint64_t)j * nsub * kLaneOut;
+        const uint32_t base = s * kFoldSub + warp * 32;
+        uint32_t v = 0;
+        if (base < nsub) {
+            const uint32_t k_end = nsub - base < 32 ? nsub - base : 32;
+            uint32_t e[32];  // all 32 sub-tiles' lane values in flight at once
 #pragma unroll
-        for (uint32_t k = 0; k < 32; ++k) e[k] = k < k_end ? tc[(uint64_t)(base + k) * kLaneOut + lane] : 0u;
+            for (uint32_t k = 0; k < 32; ++k) e[k] = k < k_end ? tc[(uint64_t)(base + k) * kLaneOut + lane] : 0u;
 #pragma unroll
-        for (uint32_t k = 0; k < 32; ++k) {
-            uint32_t x = shift32(nlt, lane4, e[k]);
+            for (uint32_t k = 0; k < 32; ++k) e[k] = shift32(nlt, lane4, e[k]);
+            // butterfly reduce-scatter: afterwards lane k holds the XOR over lanes of e[k]
+            // (31 shuffles instead of 32 x 5 for one all-reduce per sub-tile)
 #pragma unroll
-            for (int o = 16; o > 0; o >>= 1) x ^= __shfl_xor_sync(0xFFFFFFFFu, x, o);
-            if (lane == k) mine = x;
+            for (int h = 16; h > 0; h >>= 1) {
+                const bool up = lane & h;  // keep the upper half of the remaining values
+#pragma unroll
+                for (int i = 0; i < h; ++i) {
+                    const uint32_t give = up ? e[i] : e[i + h];
+                    const uint32_t keep = up ? e[i + h] : e[i];
+                    e[i] = keep ^ __shfl_xor_sync(0xFFFFFFFFu, give, h);
+                }
+            }
+            const uint32_t mine = e[0];
+            if (lane < k_end) v = multmodp(F.tile_shift[base + lane], mine);
         }
-        if (lane < k_end) v ^= multmodp(F.tile_shift[base + lane], mine);
-    }
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v ^= __shfl_xor_sync(0xFFFFFFFFu, v, o);
-    if (lane == 0) red[warp] = v;
-    __syncthreads();
-    if (threadIdx.x == 0) {
+        for (int o = 16; o > 0; o >>= 1) v ^= __shfl_xor_sync(0xFFFFFFFFu, v, o);
+        if (lane == 0) red[warp] = v;
+        __syncthreads();  // every lane-CRC word of this unit has been read
+        if (threadIdx.x == 0) {
+            uint32_t raw = 0;
+            for (int i = 0; i < kFoldThreads / 32; ++i) raw ^= red[i];
+            tc[(uint64_t)s * kFoldSub * kLaneOut] = raw;
+        }
+        __syncthreads();  // red[] reused by the next unit
+    }
+}
+
+// k_chunk_crcs: one CTA; thread t takes chunks t, t+1024, ...: XOR of the chunk's S shares ->
+// standard CRC (-> compare with the expected table) and its term of the slice digest
+// (shifted to the slice end); the digest is a block XOR-reduction.
+constexpr int kCrcThreads = 1024;
+__global__ void __launch_bounds__(kCrcThreads) k_chunk_crcs(const FinalizeParams F) {
+    __shared__ uint32_t red[kCrcThreads / 32];
+    const uint32_t S = fold_splits(F.tpc);
+    uint32_t acc = 0, nbad = 0;
+    for (uint32_t j = threadIdx.x; j < F.n; j += kCrcThreads) {
+        const uint32_t *tc = F.tile_crc + (uint64_t)j * F.tpc * kLaneOut;
         uint32_t raw = 0;
-        for (int i = 0; i < kFinThreads / 32; ++i) raw ^= red[i];
+        for (uint32_t s = 0; s < S; ++s) raw ^= tc[(uint64_t)s * kFoldSub * kLaneOut];
         const uint32_t crc = raw ^ F.ff[0] ^ 0xFFFFFFFFu;
         F.crc_out[j] = crc;
         if (F.expect) {
             const uint32_t badj = crc != F.expect[j];
             F.bad[j] = badj;
-            if (badj) atomicAdd(&F.scratch[2], 1u);
+            nbad += badj;
         }
-        atomicXor(&F.scratch[0], multmodp(F.chunk_shift[j], raw));
-        __threadfence();
-        if (atomicAdd(&F.scratch[1], 1u) == F.n - 1) {
-            __threadfence();
-            const uint32_t acc = atomicXor(&F.scratch[0], 0u);
-            F.scratch[3] = acc ^ F.ff[1] ^ 0xFFFFFFFFu;
-        }
+        acc ^= multmodp(F.chunk_shift[j], raw);
+    }
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        acc ^= __shfl_xor_sync(0xFFFFFFFFu, acc, o);
+        nbad += __shfl_xor_sync(0xFFFFFFFFu, nbad, o);
+    }
+    if (lane == 0) red[warp] = acc;
+    if (lane == 0 && nbad) atomicAdd(&F.scratch[2], nbad);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t d = 0;
+        for (int i = 0; i < kCrcThreads / 32; ++i) d ^= red[i];
+        F.scratch[3] = d ^ F.ff[1] ^ 0xFFFFFFFFu;
     }
 }
 
@@ -564,7 +655,12 @@ cudaError_t launch_unpack(const SnapParams &p, int grid, cudaStream_t s) {
 
 cudaError_t launch_finalize(const FinalizeParams &p, cudaStream_t s) {
     if (p.n == 0) return cudaSuccess;
-    k_finalize<<<p.n, kFinThreads, 0, s>>>(p);
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint32_t units = p.n * fold_splits(p.tpc);
+    k_fold_subtiles<<<units < (uint32_t)sms ? units : (uint32_t)(sms > 0 ? sms : 1), kFoldThreads, 0, s>>>(p);
+    k_chunk_crcs<<<1, kCrcThreads, 0, s>>>(p);
     return cudaGetLastError();
 }
 

@@ -44,14 +44,14 @@ struct SnapParams {
 };
 
 struct FinalizeParams {
-    const uint32_t *tile_crc;    // K1/K2's lane CRCs, tile_crc_words(tpc) per chunk
+    uint32_t *tile_crc;          // K1/K2's lane CRCs, tile_crc_words(tpc) per chunk (overwritten)
     const CrcTables *tables;     // NL (lane -> sub-tile end shifts)
     uint32_t n, tpc;             // tiles per chunk
     const uint32_t *tile_shift, *chunk_shift, *ff;
     uint32_t *crc_out;           // [n] standard CRC32C per chunk
     const uint32_t *expect;      // restore: [n] expected CRCs (nullptr when packing)
     uint32_t *bad;               // restore: [n] 1 = mismatch
-    uint32_t *scratch;           // [4] zeroed: digest accumulator, done counter, n_bad, digest out
+    uint32_t *scratch;           // [4] zeroed: unused, unused, n_bad, digest out
 };
 
 // words of K1/K2 lane-CRC output per chunk
@@ -65,6 +65,7 @@ void free_geometry(DevGeometry *g);
 int snapshot_grid(int device, uint32_t n_items, uint32_t cap);
 cudaError_t launch_pack(const SnapParams &p, int grid, cudaStream_t s);
 cudaError_t launch_unpack(const SnapParams &p, int grid, cudaStream_t s);
-cudaError_t launch_finalize(const FinalizeParams &p, cudaStream_t s);
+cudaError_t launch_finalize(const FinalizeParams &p, cudaStream_t s);  // kFinalizeLaunches kernels
+constexpr int kFinalizeLaunches = 2;
 
 }  // namespace pcc

@@ -869,7 +869,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
     F.scratch = c->scratch_dev[s];
     if (e == cudaSuccess) e = launch_finalize(F, c->pack_stream);
     cudaEventRecord(ck->ev_fin_k, c->pack_stream);
-    if (c->n) c->launches += 1;
+    if (c->n) c->launches += kFinalizeLaunches;
     cudaMemcpyAsync(c->crc_dev[s] + c->n, c->scratch_dev[s] + 3, 4, cudaMemcpyDeviceToDevice, c->pack_stream);
     cudaMemcpyAsync(c->crc_host[s], c->crc_dev[s], (c->n + 1) * sizeof(uint32_t), cudaMemcpyDeviceToHost,
                     c->pack_stream);
@@ -1193,7 +1193,7 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     F.bad = bad;
     F.scratch = scr;
     if (rc == PCC_OK && (e = launch_finalize(F, c->pack_stream))) rc = cuda_error(e, "finalize");
-    c->launches += 1;
+    c->launches += kFinalizeLaunches;
     std::vector<uint32_t> flags(n);
     uint32_t sc[4] = {0, 0, 0, 0};
     if (rc == PCC_OK) {
@@ -1363,7 +1363,7 @@ int dp_fanout(pcc_ctx *c, uint32_t slot) {
                 rc = cuda_error(e, "fanout finalize");
                 break;
             }
-            launches += 2;
+            launches += 1 + kFinalizeLaunches;
         }
         if ((e = cudaStreamSynchronize(c->pack_stream))) rc = cuda_error(e, "fanout sync");  // recv reused next group
         std::vector<uint32_t> sc(4 * W);
