@@ -49,7 +49,13 @@ int pcc_host_open(const pcc_host_config *cfg, pcc_host **out) {
     ec.n_inflight = cfg->max_inflight;
     ec.fsync = cfg->fsync != 0;
     pcc_host *raw = h.get();
-    ec.on_state = [raw](uint64_t counter, int st) { raw->states[counter] = st; };  // under engine lock
+    // called under the engine's DP lock, from whichever thread's complete() drained the in-order
+    // commits; h->mu orders it against pcc_host_begin / _state (no path holds h->mu while it
+    // calls into the engine, so the two locks never nest the other way)
+    ec.on_state = [raw](uint64_t counter, int st) {
+        std::lock_guard<std::mutex> lk(raw->mu);
+        raw->states[counter] = st;
+    };
     int rc = h->engine.open(ec);
     if (rc) return rc;
     *out = h.release();
