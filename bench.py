@@ -172,6 +172,14 @@ def load_traffic(name):
         return None
 
 
+def default_chunk_bytes(args):
+    """chunk size b (R2): 4 MiB for the 64 MiB state; 16 MiB for VGG-16 (fig14 sweep: best of
+    4/16/64/256 MiB — less zero padding in the last chunk); 64 MiB for the 10-100 GB states"""
+    if args.chunk_mib:
+        return args.chunk_mib << 20
+    return {"c1": 4 << 20, "c2": 16 << 20}.get(args.config, 64 << 20)
+
+
 def run_reference(args, rank, world):
     """--impl reference: the CPU oracle on the same workload, bounded sample per step."""
     if rank != 0:
@@ -180,7 +188,7 @@ def run_reference(args, rank, world):
     from synth import config_tensors
     import torch
     specs = config_tensors(args.config)
-    cb = 64 << 20 if args.config != "c1" else 4 << 20
+    cb = default_chunk_bytes(args)
     from synth import make_state
     state = make_state(specs, "cpu", seed=0, it=0)
     import oracle as O
@@ -188,17 +196,23 @@ def run_reference(args, rank, world):
           for t in state]
     nb = [s.nbytes for s in specs]
     off, end, c = O.layout(nb, 256, cb)
-    per_step = 1
+    # a bounded sample per step: the next `per_step` chunks of the image (about 128 MiB), packed
+    # by an oracle handed only the tensors overlapping them (its pack walks every byte it is given)
+    per_step = max(1, min(c, (128 << 20) // cb))
     times = []
     j = 0
     for step in range(args.warmup + args.steps):
+        a = j % c
+        k = min(per_step, c - a)
+        lo, hi = a * cb, (a + k) * cb
+        mine = {i: hb[i] for i in range(len(nb)) if int(off[i]) < hi and int(off[i]) + nb[i] > lo and nb[i]}
         t0 = time.perf_counter()
-        img = O.pack(hb, 256, cb, first_chunk=j % c, count=min(per_step, c - j % c))
+        img = O.pack_chunks_sparse(nb, mine, 256, cb, a, k)
         O.chunk_crcs(img, cb)
         dt = time.perf_counter() - t0
         if step >= args.warmup:
             times.append((img.nbytes, dt))
-        j += per_step
+        j += k
     tot_b = sum(b for b, _ in times)
     tot_t = sum(t for _, t in times)
     v = tot_b / tot_t / 1e9
@@ -209,7 +223,8 @@ def run_reference(args, rank, world):
             "config": {"workload": WORKLOADS.get(args.config, args.config), "config": args.config,
                        "chunk_bytes": cb},
             "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle",
-                             "sample": f"per step: pack + CRC32C of {per_step} {cb >> 20} MiB chunks"},
+                             "sample": f"per step: pack + CRC32C of the next {per_step} {cb >> 20} MiB chunks of the image "
+                                       f"(1 thread, plain C)"},
             "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -257,9 +272,7 @@ def main():
     from synth import config_tensors, make_state
 
     specs = config_tensors(args.config)
-    # chunk size b (R2): 4 MiB for the 64 MiB state; 16 MiB for VGG-16 (fig14 sweep: best of
-    # 4/16/64/256 MiB — less zero padding in the last chunk); 64 MiB for the 10-100 GB states
-    cb = args.chunk_mib << 20 if args.chunk_mib else {"c1": 4 << 20, "c2": 16 << 20}.get(args.config, 64 << 20)
+    cb = default_chunk_bytes(args)
     state = make_state(specs, "cuda", seed=0, it=0)
     state_bytes = sum(s.nbytes for s in specs)
     uid = None
@@ -348,7 +361,8 @@ def main():
     launches = ck.kernel_launches() - launches0
     clk = clocks.stop()
     infos = [ck.info(h) for h in hs]
-    pack_ms = statistics.mean(i["pack_ms"] for i in infos)
+    pack_ms = statistics.mean(i["pack_ms"] for i in infos)  # U-gate span (incl. ring waits between launches)
+    k1_ms = statistics.mean(i["k1_busy_ms"] for i in infos)  # K1's own launches, summed per checkpoint
     fin_ms = statistics.mean(i["finalize_ms"] for i in infos)
     lat_ms = statistics.median((i["t_committed_us"] - i["t_call_us"]) / 1e3 for i in infos)
     t = torch.tensor([dev_ms], device="cpu" if args.share_gpu else "cuda")
@@ -432,7 +446,7 @@ def main():
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
             peaks = json.load(f)
         k1_bytes = 2 * slice_bytes  # read the slice's state bytes + write the packed slice (R3: pads count)
-        k1_achieved = k1_bytes / (pack_ms * 1e-3) / 1e9
+        k1_achieved = k1_bytes / (k1_ms * 1e-3) / 1e9
         link_achieved = slice_bytes / (ms_total * 1e-3 / args.steps) / 1e9
         cpu = cpu_all = None
         if not args.no_cpu_baseline and args.config in ("c1", "c2", "c3"):
@@ -458,7 +472,9 @@ def main():
             "roofline": {"bound": "hbm", "kernel": "k_snapshot<pack> (K1)", "achieved": k1_achieved,
                          "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": k1_achieved / peaks["hbm_gbs"],
                          "traffic": load_traffic(f"{args.config}_k1"),
-                         "algorithmic_bytes_per_launch": k1_bytes, "launch_ms": pack_ms,
+                         "algorithmic_bytes_per_checkpoint": k1_bytes, "k1_ms_per_checkpoint": k1_ms,
+                         "k1_launches_per_checkpoint": (launches - 2 * args.steps) / args.steps,  # minus the 2 finalize kernels
+                         "pack_span_ms": pack_ms,
                          "peak_source": "MEASURED_PEAKS.json hbm_gbs (burst copy)"},
             "link_roofline": {"bound": "pcie_d2h", "achieved": link_achieved, "peak": peak_link, "unit": "GB/s",
                               "frac": link_achieved / peak_link,

@@ -155,8 +155,10 @@ typedef struct {
     double t_landed_us;        /*   last chunk landed in host memory                                */
     double t_persisted_us;     /*   last chunk persisted                                            */
     double t_committed_us;     /*   local commit                                                    */
-    float pack_ms;             /* CUDA-event time of K1 (all launches of this checkpoint)           */
-    float finalize_ms;         /* CUDA-event time of the CRC finalize kernel                       */
+    float pack_ms;             /* CUDA-event span of K1: first launch start -> last launch end      */
+                               /*   (the U-gate span; includes waits for ring space between launches) */
+    float finalize_ms;         /* CUDA-event time of the CRC finalize kernels                      */
+    float k1_busy_ms;          /* sum of the K1 launches' own CUDA-event durations                 */
 } pcc_ckpt_info;
 
 /* Opens (creates) the checkpoint file, allocates staging / HBM ring, starts the persist

@@ -53,7 +53,8 @@ class Info(C.Structure):
     _fields_ = [("iter", C.c_uint64), ("counter", C.c_uint64), ("slot", C.c_uint32), ("state", C.c_uint32),
                 ("digest", C.c_uint32), ("n_chunks", C.c_uint32), ("t_call_us", C.c_double),
                 ("t_packed_us", C.c_double), ("t_landed_us", C.c_double), ("t_persisted_us", C.c_double),
-                ("t_committed_us", C.c_double), ("pack_ms", C.c_float), ("finalize_ms", C.c_float)]
+                ("t_committed_us", C.c_double), ("pack_ms", C.c_float), ("finalize_ms", C.c_float),
+                ("k1_busy_ms", C.c_float)]
 
 
 class HostConfig(C.Structure):

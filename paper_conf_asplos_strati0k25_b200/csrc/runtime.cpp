@@ -87,7 +87,10 @@ struct Ckpt {
     std::atomic<uint32_t> remaining{0};
     cudaEvent_t ev_train = nullptr, ev_begin = nullptr, ev_packed = nullptr, ev_fin_k = nullptr, ev_final = nullptr;
     double t_call = 0, t_packed = 0, t_landed = 0, t_persisted = 0, t_committed = 0;
-    float pack_ms = 0, fin_ms = 0;
+    float pack_ms = 0, fin_ms = 0, k1_busy_ms = 0;
+    // timing events around every K1 launch: the kernel's busy time, without the gaps in which
+    // the host waits for ring space between launches (those count in pack_ms, the U-gate span)
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> k1_ev;
     uint32_t digest = 0;
     std::vector<uint32_t> crc;
 };
@@ -217,6 +220,15 @@ struct pcc_ctx {
 
 namespace {
 
+// a timing event pair for one K1 launch of ck (destroyed with the checkpoint's events)
+std::pair<cudaEvent_t, cudaEvent_t> k1_events(Ckpt *ck) {
+    std::pair<cudaEvent_t, cudaEvent_t> p{nullptr, nullptr};
+    cudaEventCreate(&p.first);
+    cudaEventCreate(&p.second);
+    ck->k1_ev.push_back(p);
+    return p;
+}
+
 cudaEvent_t get_event(pcc_ctx *c) {
     {
         std::lock_guard<std::mutex> lk(c->evpool_mu);
@@ -303,6 +315,11 @@ void finish_ckpt(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
     cudaError_t e = cudaEventSynchronize(ck->ev_final);
     if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "finalize"));
     cudaEventElapsedTime(&ck->pack_ms, ck->ev_begin, ck->ev_packed);
+    ck->k1_busy_ms = 0;
+    for (auto &p : ck->k1_ev) {
+        float ms = 0;
+        if (cudaEventElapsedTime(&ms, p.first, p.second) == cudaSuccess) ck->k1_busy_ms += ms;
+    }
     cudaEventElapsedTime(&ck->fin_ms, ck->ev_packed, ck->ev_fin_k);  // the finalize kernel alone
     const uint32_t *h = c->crc_host[ck->t.slot];
     ck->crc.assign(h, h + c->n);
@@ -488,6 +505,11 @@ void destroy_ckpt_events(pcc_ctx *c, Ckpt *ck) {
     cudaEventDestroy(ck->ev_final);
     for (auto &L : ck->launches) put_event(c, L.ev);
     ck->launches.clear();
+    for (auto &p : ck->k1_ev) {
+        cudaEventDestroy(p.first);
+        cudaEventDestroy(p.second);
+    }
+    ck->k1_ev.clear();
 }
 
 // keeps the newest kKeep terminal records queryable (pcc_info), frees older ones
@@ -808,7 +830,10 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
         P.ring_head = 0;
         P.ring_slots = c->n ? c->n : 1;
         cudaEventRecord(ck->ev_begin, c->pack_stream);
+        const auto k1e = k1_events(ck.get());
+        cudaEventRecord(k1e.first, c->pack_stream);
         e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas), c->pack_stream);
+        cudaEventRecord(k1e.second, c->pack_stream);
         c->launches += c->n ? 1 : 0;
         cudaEvent_t ev = get_event(c);
         cudaEventRecord(ev, c->pack_stream);
@@ -828,8 +853,14 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
         while (done < c->n && e == cudaSuccess) {
             uint64_t k;
             {
+                // launch windows of at least a quarter ring (or the rest of the slice): when the
+                // link is the bottleneck the ring frees a chunk or two at a time, and a K1 launch
+                // per freed chunk pays the table load and launch latency each time (C3 with
+                // N = 4 over a 2-slice ring: 114 launches per checkpoint, 11.7 ms of K1 instead
+                // of 5.7).  The chunks already packed keep the copy engine busy meanwhile.
+                const uint64_t want = std::min<uint64_t>(c->n - done, std::max<uint64_t>(1, c->ring_slots / 4));
                 std::unique_lock<std::mutex> lk(c->ring_mu);
-                c->ring_cv.wait(lk, [&] { return c->ring_tail + c->ring_slots > ck->ring_start + done; });
+                c->ring_cv.wait(lk, [&] { return c->ring_tail + c->ring_slots >= ck->ring_start + done + want; });
                 k = std::min<uint64_t>(c->n - done, c->ring_tail + c->ring_slots - (ck->ring_start + done));
             }
             P.first = (uint32_t)done;
@@ -838,7 +869,10 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
             P.ring_head = ck->ring_start % c->ring_slots;
             P.ring_slots = c->ring_slots;
             if (done == 0) cudaEventRecord(ck->ev_begin, c->pack_stream);  // K1 time excludes ring waits
+            const auto k1e = k1_events(ck.get());
+            cudaEventRecord(k1e.first, c->pack_stream);
             e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas), c->pack_stream);
+            cudaEventRecord(k1e.second, c->pack_stream);
             c->launches += 1;
             cudaEvent_t ev = get_event(c);
             cudaEventRecord(ev, c->pack_stream);
@@ -1012,6 +1046,7 @@ int pcc_info(pcc_ctx *c, pcc_handle h, pcc_ckpt_info *info, uint32_t *crc, uint3
         info->t_committed_us = ck->t_committed;
         info->pack_ms = ck->pack_ms;
         info->finalize_ms = ck->fin_ms;
+        info->k1_busy_ms = ck->k1_busy_ms;
         if (crc)
             for (uint32_t i = 0; i < crc_cap && i < ck->crc.size(); ++i) crc[i] = ck->crc[i];
     }
