@@ -117,6 +117,35 @@ def d2h_peak_gbs(torch, nbytes=1 << 30):
     return nbytes / (best * 1e-3) / 1e9
 
 
+def bidir_peak_gbs(torch, nbytes=1 << 30):
+    """Pinned H2D and D2H copies of `nbytes` each running at once (separate streams): GB/s per
+    direction.  The e2e line moves the slice up AND the checkpoint down every step, so this, not
+    the one-way peak, bounds it."""
+    d1 = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    d2 = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    h1 = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    h2 = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    best = 1e9
+    for i in range(4):
+        torch.cuda.synchronize()
+        a = torch.cuda.Event(enable_timing=True)
+        b1, b2 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(s1)
+        s2.wait_event(a)
+        with torch.cuda.stream(s1):
+            d1.copy_(h1, non_blocking=True)
+        with torch.cuda.stream(s2):
+            h2.copy_(d2, non_blocking=True)
+        b1.record(s1)
+        b2.record(s2)
+        torch.cuda.synchronize()
+        if i >= 1:
+            best = min(best, max(a.elapsed_time(b1), a.elapsed_time(b2)))
+    del d1, d2, h1, h2
+    return nbytes / (best * 1e-3) / 1e9
+
+
 def cpu_baseline(specs, state, cb, budget_bytes=2 << 30, threads=1, hb=None):
     """The oracle as it stands (plain C: byte-loop pack + byte-at-a-time CRC32C) on a bounded
     sample: pack calls over the first chunks of the same image, up to `budget_bytes` (the whole
@@ -337,8 +366,14 @@ def main():
     clocks.start()
     time.sleep(0.5)
     # ---- warm-up
+    warm = []
     for _ in range(args.warmup):
-        ck.wait(one_ckpt())
+        h = one_ckpt()
+        ck.wait(h)
+        warm.append(ck.info(h))
+    # one checkpoint at a time with nothing else running (SURVEY §8(d) "idle"): K1 start -> last
+    # chunk landed, GPU clock; the first warm-up checkpoint also pays first-touch costs
+    idle_ms = statistics.median(i["snapshot_ms"] for i in warm[1:] or warm)
     if world > 1:
         ck.commit()
     barrier()
@@ -415,6 +450,7 @@ def main():
         restore = {"iter": rit, "ms": rdt * 1e3, "gbs": state_bytes / rdt / 1e9, "bad_chunks": len(rbad),
                    "path": "file mapping -> H2D into the HBM ring -> K2 verify+scatter"}
     peak_link = d2h_peak_gbs(torch)
+    peak_bidir = bidir_peak_gbs(torch)
     ck.close()
     if path and os.path.exists(path):
         os.unlink(path)
@@ -469,6 +505,9 @@ def main():
                        else "null sink", "l2": "inputs larger than L2 (state >> 126 MB)"},
             "per_gpu_gbs": value / world,
             "checkpoint_latency_ms_p50": lat_ms,
+            "snapshot_idle": {"ms": idle_ms, "gbs": state_bytes / (idle_ms * 1e-3) / 1e9,
+                              "def": "K1 start -> last chunk landed in host memory, CUDA events, one checkpoint "
+                                     "in flight, median of the warm-up checkpoints after the first"},
             "roofline": {"bound": "hbm", "kernel": "k_snapshot<pack> (K1)", "achieved": k1_achieved,
                          "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": k1_achieved / peaks["hbm_gbs"],
                          "traffic": load_traffic(f"{args.config}_k1"),
@@ -484,7 +523,10 @@ def main():
             "cpu_baseline": cpu,
             "cpu_baseline_all_cores": cpu_all,
             "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": h2d_bytes,
-                    "d2h_bytes_per_step": slice_bytes + 4 * (geo["count"] + 1)},
+                    "d2h_bytes_per_step": slice_bytes + 4 * (geo["count"] + 1),
+                    # both directions busy every step: the bound is the concurrent H2D + D2H rate
+                    "link_peak_bidir_gbs_per_direction": peak_bidir,
+                    "frac_of_bidir": e2e_value / peak_bidir},
             "gpu_launches": launches,
             "clocks": clk,
             "slowdown": slowdown,

@@ -159,6 +159,7 @@ typedef struct {
                                /*   (the U-gate span; includes waits for ring space between launches) */
     float finalize_ms;         /* CUDA-event time of the CRC finalize kernels                      */
     float k1_busy_ms;          /* sum of the K1 launches' own CUDA-event durations                 */
+    float snapshot_ms;         /* CUDA-event time from K1's start to the last chunk's D2H end      */
 } pcc_ckpt_info;
 
 /* Opens (creates) the checkpoint file, allocates staging / HBM ring, starts the persist

@@ -36,6 +36,16 @@ PCC_API int pcc_k_unpack(const pcc_tensor *t, uint32_t n, uint32_t align, uint64
                  uint64_t count, const void *src, const uint32_t *expect, uint32_t *bad, uint32_t *n_bad,
                  uint32_t *digest, void *stream);
 
+/* Transport self-test of the commit collective (C1 of SURVEY §2.3; §4.1, reading
+ * R9): a one-rank NCCL communicator on `device` runs the calls the commit and restore paths
+ * issue over the library's own communicator — ncclAllReduce of int64 with MIN and with MAX on
+ * vals[n] (HOST arrays; out_min / out_max receive the reduced vectors, equal to vals with one
+ * rank) and ncclAllGather of bytes (*gather_ok = 1 when the gathered bytes equal the sent
+ * ones).  For tests: one GPU cannot host two NCCL ranks.  -PCC_ENCCL when libnccl.so.2 cannot
+ * be loaded or a call fails, -PCC_ECUDA on a CUDA error. */
+PCC_API int pcc_k_nccl_selftest(int device, const int64_t *vals, uint32_t n, int64_t *out_min, int64_t *out_max,
+                                uint32_t *gather_ok);
+
 /* Layout queries (host only, no GPU needed): image offsets of the n tensors and the chunk
  * count C for this registration. */
 PCC_API int pcc_k_layout(const pcc_tensor *t, uint32_t n, uint32_t align, uint64_t chunk_bytes, uint64_t *off,

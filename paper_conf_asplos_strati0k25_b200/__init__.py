@@ -54,7 +54,7 @@ class Info(C.Structure):
                 ("digest", C.c_uint32), ("n_chunks", C.c_uint32), ("t_call_us", C.c_double),
                 ("t_packed_us", C.c_double), ("t_landed_us", C.c_double), ("t_persisted_us", C.c_double),
                 ("t_committed_us", C.c_double), ("pack_ms", C.c_float), ("finalize_ms", C.c_float),
-                ("k1_busy_ms", C.c_float)]
+                ("k1_busy_ms", C.c_float), ("snapshot_ms", C.c_float)]
 
 
 class HostConfig(C.Structure):
@@ -90,6 +90,8 @@ _SIGS = {
     "pcc_k_unpack": (C.c_int, [C.POINTER(Tensor), C.c_uint32, C.c_uint32, C.c_uint64, C.c_uint64, C.c_uint64,
                                _P, _P, _P, _P, _P, _P]),
     "pcc_k_layout": (C.c_int, [C.POINTER(Tensor), C.c_uint32, C.c_uint32, C.c_uint64, _u64p, _u64p, _u64p]),
+    "pcc_k_nccl_selftest": (C.c_int, [C.c_int, C.POINTER(C.c_int64), C.c_uint32, C.POINTER(C.c_int64),
+                                      C.POINTER(C.c_int64), C.POINTER(C.c_uint32)]),
     "pcc_host_open": (C.c_int, [C.POINTER(HostConfig), C.POINTER(C.c_void_p)]),
     "pcc_host_begin": (C.c_int, [_P, C.c_uint64, _u64p, _u32p]),
     "pcc_host_filling": (C.c_int, [_P, C.c_uint64]),
@@ -329,6 +331,15 @@ def nccl_unique_id():
 
 
 # ------------------------------------------------------------------- kernel-level calls
+def nccl_selftest(vals, device=0):
+    """The commit collective's NCCL calls on a one-rank communicator: (min, max, gather_ok)."""
+    n = len(vals)
+    v = (C.c_int64 * n)(*vals)
+    mn, mx, ok = (C.c_int64 * n)(), (C.c_int64 * n)(), C.c_uint32()
+    _check(_lib.pcc_k_nccl_selftest(device, v, n, mn, mx, C.byref(ok)), "pcc_k_nccl_selftest")
+    return list(mn), list(mx), bool(ok.value)
+
+
 def k_layout(tensors, align=256, chunk_bytes=4 << 20):
     tab, keep = tensor_table(tensors)
     n = len(tensors)

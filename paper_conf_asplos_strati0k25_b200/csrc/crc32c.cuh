@@ -57,10 +57,11 @@ __host__ __device__ inline uint32_t x8n(const uint32_t *x2n, uint64_t n) {
 }
 
 // ---------------------------------------------------------------- kernel geometry
-// One CTA of 32 warps per SM (all warps share one copy of the tables); the work item is an
-// 8 KiB tile of one chunk, owned by one warp = 8 rounds of 1 KiB.  In round r lane l owns the 32 bytes at
+// One CTA per SM (all warps share one copy of the tables); the work item is an 8 KiB tile of
+// one chunk, owned by one warp = 8 rounds of 1 KiB.  In round r lane l owns the 32 bytes at
 // warp_base + r*1024 + 32*l: one 256-bit load and one 256-bit store per lane, so every warp
-// access is 1 KiB contiguous.  Loads run kAhead rounds ahead in registers.  Per round:
+// access is 1 KiB contiguous.  Loads run kAheadOf<> rounds ahead in registers, and the round
+// after those is prefetched into L2 (kPf2Of<>).  Per round:
 //     x = shift(s, 992);  s = raw16(w0 ^ x);  s = raw16(w1 ^ s)
 // (feeding a 16-byte word into register r equals raw16 of the word with its first 4 bytes
 // XOR r).  After the last round every lane writes its register (relative to the end of its
@@ -76,20 +77,43 @@ __host__ __device__ inline uint32_t x8n(const uint32_t *x2n, uint64_t n) {
 // gets a table of only its own 2^bits values.  (Byte-indexed slicing-by-16 tables cost 20
 // lookups per 16 B, but random indices collide in banks ~2.9-way on average; ncu showed the
 // L1/shared pipe at 81% with that design, K1 at 0.45 of HBM.)
-#ifndef PCC_KWARPS
-#define PCC_KWARPS 32
+// Warps per CTA and rounds of loads held in registers ahead of the CRC, per direction (K1 packs,
+// K2 unpacks; measured in DESIGN.md §6: K1 prefers 32 warps x 1 round, K2 28 warps x 2 rounds).
+// A/B builds override them with -DPCC_KWARPS_PACK=... etc.
+#ifndef PCC_KWARPS_PACK
+#define PCC_KWARPS_PACK 32
 #endif
-constexpr int kWarps = PCC_KWARPS;                   // warps per CTA (A/B builds: -DPCC_KWARPS)
-constexpr int kThreads = kWarps * 32;
+#ifndef PCC_KAHEAD_PACK
+#define PCC_KAHEAD_PACK 1
+#endif
+#ifndef PCC_KWARPS_UNPACK
+#define PCC_KWARPS_UNPACK 28
+#endif
+#ifndef PCC_KAHEAD_UNPACK
+#define PCC_KAHEAD_UNPACK 2
+#endif
+// Per-lane L2 prefetch of the round after the ones in registers (no registers): K1 +2-3.5%;
+// K2 at 28 warps x 2 rounds loses 4% with it (ncu 400 -> 416 us), so only K1 uses it
+#ifndef PCC_PF2_PACK
+#define PCC_PF2_PACK 1
+#endif
+#ifndef PCC_PF2_UNPACK
+#define PCC_PF2_UNPACK 0
+#endif
+// K1 also prefetches the first rounds of a warp's next item during its last rounds (+1.5-2%)
+#ifndef PCC_XPF
+#define PCC_XPF 1
+#endif
+constexpr bool kXpf = PCC_XPF != 0;
+template <bool kPack> constexpr int kWarpsOf = kPack ? PCC_KWARPS_PACK : PCC_KWARPS_UNPACK;
+template <bool kPack> constexpr int kThreadsOf = kWarpsOf<kPack> * 32;
+template <bool kPack> constexpr int kAheadOf = kPack ? PCC_KAHEAD_PACK : PCC_KAHEAD_UNPACK;
+template <bool kPack> constexpr bool kPf2Of = kPack ? PCC_PF2_PACK != 0 : PCC_PF2_UNPACK != 0;
 constexpr int kWpl = 2;                              // 16-byte words per lane per round
 constexpr uint32_t kLaneSpan = 16 * kWpl;            // 32 B
 constexpr uint32_t kRound = 32 * kLaneSpan;          // 1 KiB per warp per round
 constexpr uint32_t kWarpBytes = 8192;                // 8 KiB per warp per tile
 constexpr int kRounds = kWarpBytes / kRound;         // 8
-#ifndef PCC_KAHEAD
-#define PCC_KAHEAD 1
-#endif
-constexpr int kAhead = PCC_KAHEAD;                   // rounds loaded ahead of the CRC (A/B builds: -DPCC_KAHEAD)
 #ifndef PCC_KRUN
 #define PCC_KRUN 1
 #endif
@@ -130,7 +154,6 @@ static_assert(kK1TableBytes + 1024 <= 227 * 1024, "K1 shared memory");
 // Constants that do not need a table.
 struct CrcConsts {
     uint32_t x2n[kX2n];
-    uint32_t warp_shift[kWarps];  // x8n((kWarps-1-w) * kWarpBytes)
     uint32_t x8n_stride;          // x8n(32*16): generic (ragged-tile) path, one warp stride
 };
 

@@ -2,11 +2,13 @@
 #include <cuda_runtime.h>
 
 #include <cstring>
+#include <vector>
 
 #include "../../include/pccheck_kernels.h"
 #include "errors.hpp"
 #include "kernels.hpp"
 #include "layout.hpp"
+#include "nccl_shim.hpp"
 
 namespace pcc {
 int cuda_error(cudaError_t e, const char *what);  // runtime.cpp
@@ -102,7 +104,7 @@ extern "C" int pcc_k_pack(const pcc_tensor *t, uint32_t n, uint32_t align, uint6
     P.ring_base = static_cast<char *>(dst);
     int dev = 0;
     cudaGetDevice(&dev);
-    cudaError_t e = launch_pack(P, snapshot_grid(dev, (uint32_t)(count * P.tpc), 0), s);
+    cudaError_t e = launch_pack(P, snapshot_grid(dev, (uint32_t)(count * P.tpc), 0, true), s);
     if (e != cudaSuccess) return cuda_error(e, "K1 launch");
     FinalizeParams F{};
     F.tile_crc = S.tile_crc;
@@ -134,7 +136,7 @@ extern "C" int pcc_k_unpack(const pcc_tensor *t, uint32_t n, uint32_t align, uin
     if ((e = cudaMalloc(&S.crc_tmp, count * sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "crc tmp");
     int dev = 0;
     cudaGetDevice(&dev);
-    e = launch_unpack(P, snapshot_grid(dev, (uint32_t)(count * P.tpc), 0), s);
+    e = launch_unpack(P, snapshot_grid(dev, (uint32_t)(count * P.tpc), 0, false), s);
     if (e != cudaSuccess) return cuda_error(e, "K2 launch");
     FinalizeParams F{};
     F.tile_crc = S.tile_crc;
@@ -153,4 +155,50 @@ extern "C" int pcc_k_unpack(const pcc_tensor *t, uint32_t n, uint32_t align, uin
     cudaMemcpyAsync(digest, S.scratch + 3, 4, cudaMemcpyDeviceToDevice, s);
     if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return cuda_error(e, "K2");
     return PCC_OK;
+}
+
+extern "C" int pcc_k_nccl_selftest(int device, const int64_t *vals, uint32_t n, int64_t *out_min, int64_t *out_max,
+                                   uint32_t *gather_ok) {
+    if (!vals || !out_min || !out_max || !gather_ok || n == 0 || n > 64) return set_error(PCC_EINVAL, "args");
+    cudaError_t e = cudaSetDevice(device);
+    if (e != cudaSuccess) return cuda_error(e, "set device");
+    uint8_t uid[128];
+    int rc = pcc_nccl_unique_id_impl(uid);
+    if (rc) return rc;
+    NcclComm comm;
+    if ((rc = comm.init(uid, 1, 0))) return rc;
+    int64_t *dev = nullptr, *pinned = nullptr;
+    uint8_t *send = nullptr, *recv = nullptr;
+    cudaStream_t s = nullptr;
+    const size_t gb = 4096;
+    std::vector<uint8_t> pat(gb), back(gb);
+    for (size_t i = 0; i < gb; ++i) pat[i] = (uint8_t)(i * 131 + 7);
+    if ((e = cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking)) || (e = cudaMalloc(&dev, 64 * sizeof(int64_t))) ||
+        (e = cudaMallocHost(&pinned, 64 * sizeof(int64_t))) || (e = cudaMalloc(&send, gb)) || (e = cudaMalloc(&recv, gb)))
+        rc = cuda_error(e, "selftest alloc");
+    if (!rc) {
+        std::memcpy(out_min, vals, n * sizeof(int64_t));
+        rc = comm.allreduce_i64(out_min, n, NcclComm::kMin, dev, pinned, s);
+    }
+    if (!rc) {
+        std::memcpy(out_max, vals, n * sizeof(int64_t));
+        rc = comm.allreduce_i64(out_max, n, NcclComm::kMax, dev, pinned, s);
+    }
+    if (!rc) {
+        cudaMemcpyAsync(send, pat.data(), gb, cudaMemcpyHostToDevice, s);
+        cudaMemsetAsync(recv, 0, gb, s);
+        rc = comm.allgather(send, recv, gb, s);
+        if (!rc) {
+            cudaMemcpyAsync(back.data(), recv, gb, cudaMemcpyDeviceToHost, s);
+            if ((e = cudaStreamSynchronize(s))) rc = cuda_error(e, "selftest sync");
+            *gather_ok = !rc && std::memcmp(back.data(), pat.data(), gb) == 0;
+        }
+    }
+    comm.destroy();
+    if (send) cudaFree(send);
+    if (recv) cudaFree(recv);
+    if (dev) cudaFree(dev);
+    if (pinned) cudaFreeHost(pinned);
+    if (s) cudaStreamDestroy(s);
+    return rc;
 }

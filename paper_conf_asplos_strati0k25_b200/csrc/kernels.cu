@@ -80,7 +80,6 @@ __global__ void k_build_tables(CrcTables *tb, CrcConsts *cs) {
         tb->NL[e] = multmodp(x8n(x2n, kLaneRun * (31 - l)), (uint32_t)((uint64_t)v << (5 * g)));
     }
     if (t < kX2n) cs->x2n[t] = x2n[t];
-    if (t < kWarps) cs->warp_shift[t] = x8n(x2n, (uint64_t)(kWarps - 1 - t) * kWarpBytes);
     if (t == 0) cs->x8n_stride = x8n(x2n, 32 * 16);
 }
 
@@ -227,6 +226,10 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
+__device__ __forceinline__ void prefetch_l2(uint64_t addr) {
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(addr));
+}
+
 struct Span {  // one lane's 32 bytes of a round
     uint4 a, b;
 };
@@ -279,7 +282,8 @@ __device__ __forceinline__ void scatter_span(RowCursor &rc, uint32_t p, const Sp
 // One warp, one 8 KiB tile: 8 rounds of 1 KiB, lane l moves the 32 bytes at 32*l of each round.
 template <bool kPack>
 __device__ __forceinline__ void tile_fast(const char *ntab, const char *nf, char *chunk, const SegRow *rows, int nrows,
-                                          uint32_t tile0, uint32_t lane, uint32_t *crc_out) {
+                                          uint32_t tile0, uint32_t lane, uint32_t *crc_out, const SegRow *next_rows,
+                                          int next_nrows, uint32_t next_tile0) {
     const uint32_t lane4 = lane * 4;
     const uint32_t wbase = tile0 + lane * kLaneRun;
     // chunk position of round r (compile-time offset once unrolled)
@@ -287,6 +291,7 @@ __device__ __forceinline__ void tile_fast(const char *ntab, const char *nf, char
     RowCursor rc;
     rc.init(rows, 0, nrows, wbase);
     auto load = [&](int r) -> Span { return kPack ? gather_span(rc, pos(r)) : ld_span(chunk + pos(r)); };
+    constexpr int kAhead = kAheadOf<kPack>;
     Span buf[kAhead + 1];
 #pragma unroll
     for (int r = 0; r < kAhead; ++r) buf[r] = load(r);
@@ -294,6 +299,25 @@ __device__ __forceinline__ void tile_fast(const char *ntab, const char *nf, char
 #pragma unroll
     for (int r = 0; r < kRounds; ++r) {
         if (r + kAhead < kRounds) buf[(r + kAhead) % (kAhead + 1)] = load(r + kAhead);
+        // warm L2 with the round after the ones in registers: its load then waits out L2, not
+        // HBM, latency (positions still reach the cursor in increasing order)
+        if (kPf2Of<kPack> && r + kAhead + 1 < kRounds) {
+            if (kPack) {
+                uint64_t a = 0;
+                if (rc.at(pos(r + kAhead + 1), a)) prefetch_l2(a);
+            } else {
+                prefetch_l2(reinterpret_cast<uint64_t>(chunk + pos(r + kAhead + 1)));
+            }
+        }
+        // ... and, in K1's last rounds, the first rounds of the warp's next item (its cursor
+        // is free once this tile's last load is out)
+        if (kPack && kXpf && next_rows && r + kAhead + 1 >= kRounds) {
+            const int q = r + kAhead + 1 - kRounds;  // round of the next tile
+            if (q == 0) rc.init(next_rows, 0, next_nrows, next_tile0 + lane * kLaneRun);  // this tile's loads are out
+            uint64_t a = 0;
+            const uint32_t np = next_tile0 + lane * kLaneRun + (q / kRun) * (kRun * kRound) + (q % kRun) * kLaneSpan;
+            if (q <= kAhead && rc.at(np, a)) prefetch_l2(a);
+        }
         Span &w = buf[r % (kAhead + 1)];
         if (kPack) st_span(chunk + pos(r), w);
 #ifdef PCC_EXP_NOCRC  // timing experiment only: the copy without the CRC (wrong CRCs)
@@ -415,13 +439,14 @@ __device__ __forceinline__ void prefetch_item(const SnapParams &P, uint32_t item
 // over the items independently (no block barrier after the table load), each fetching its
 // next tile's row descriptor one tile ahead.
 template <bool kPack>
-__global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
+__global__ void __launch_bounds__(kThreadsOf<kPack>, 1) k_snapshot(const SnapParams P) {
     extern __shared__ __align__(128) uint8_t smem[];  // NT + NF (kK1TableBytes)
     const char *ntab = reinterpret_cast<const char *>(smem);
     const char *nf = ntab + kNtBytes;
     __shared__ __align__(8) uint64_t tbar;
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t n_items = P.count * P.tpc;
+    constexpr int kWarps = kWarpsOf<kPack>;
     const uint32_t stride = gridDim.x * kWarps;
     uint32_t item = blockIdx.x * kWarps + (threadIdx.x >> 5);
     // 256-bit accesses need 32-B aligned chunks (chunk_bytes is only required to be a multiple
@@ -446,7 +471,9 @@ __global__ void __launch_bounds__(kThreads, 1) k_snapshot(const SnapParams P) {
         uint32_t *crc_out = P.tile_crc + ((uint64_t)j * P.tpc + t) * kLaneOut;
         const SegRow *rows = P.rows + tr.x;
         if (rem >= kTile && fast_ok)
-            tile_fast<kPack>(ntab, nf, chunk, rows, (int)tr.y, tile0, lane, crc_out);
+            tile_fast<kPack>(ntab, nf, chunk, rows, (int)tr.y, tile0, lane, crc_out,
+                             item + stride < n_items ? P.rows + trn.x : nullptr, (int)trn.y,
+                             ((item + stride) % P.tpc) * kTile);
         else
             tile_generic<kPack>(P, ntab, chunk, rows, (int)tr.y, tile0, rem < kTile ? (uint32_t)rem : kTile, lane,
                                 crc_out);
@@ -619,37 +646,39 @@ void free_geometry(DevGeometry *g) {
     g->tile_shift = g->chunk_shift = g->ff = nullptr;
 }
 
+template <bool kPack>
 static int resident_ctas(int device) {
     static int cached[64] = {};
     if (device < 0 || device >= 64) return 1;
     if (!cached[device]) {
         int per_sm = 0, sms = 0;
-        cudaFuncSetAttribute(k_snapshot<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, kK1TableBytes);
-        cudaFuncSetAttribute(k_snapshot<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, kK1TableBytes);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snapshot<true>, kThreads, kK1TableBytes);
+        cudaFuncSetAttribute(k_snapshot<kPack>, cudaFuncAttributeMaxDynamicSharedMemorySize, kK1TableBytes);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snapshot<kPack>, kThreadsOf<kPack>, kK1TableBytes);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
         cached[device] = (per_sm > 0 ? per_sm : 1) * (sms > 0 ? sms : 1);
     }
     return cached[device];
 }
 
-int snapshot_grid(int device, uint32_t n_items, uint32_t cap) {  // n_items = 8 KiB tiles (one warp each)
-    int g = resident_ctas(device);
+// n_items = 8 KiB tiles (one warp each)
+int snapshot_grid(int device, uint32_t n_items, uint32_t cap, bool pack) {
+    int g = pack ? resident_ctas<true>(device) : resident_ctas<false>(device);
     if (cap && (int)cap < g) g = (int)cap;
-    const uint32_t need = (n_items + kWarps - 1) / kWarps;
+    const uint32_t w = pack ? kWarpsOf<true> : kWarpsOf<false>;
+    const uint32_t need = (n_items + w - 1) / w;
     if ((uint32_t)g > need) g = (int)need;
     return g < 1 ? 1 : g;
 }
 
 cudaError_t launch_pack(const SnapParams &p, int grid, cudaStream_t s) {
     if (p.count == 0) return cudaSuccess;
-    k_snapshot<true><<<grid, kThreads, kK1TableBytes, s>>>(p);
+    k_snapshot<true><<<grid, kThreadsOf<true>, kK1TableBytes, s>>>(p);
     return cudaGetLastError();
 }
 
 cudaError_t launch_unpack(const SnapParams &p, int grid, cudaStream_t s) {
     if (p.count == 0) return cudaSuccess;
-    k_snapshot<false><<<grid, kThreads, kK1TableBytes, s>>>(p);
+    k_snapshot<false><<<grid, kThreadsOf<false>, kK1TableBytes, s>>>(p);
     return cudaGetLastError();
 }
 

@@ -62,7 +62,7 @@ cudaError_t device_tables(int device, const CrcTables **tables, const CrcConsts 
 cudaError_t setup_geometry(DevGeometry *g, uint64_t chunk_bytes, uint32_t n, cudaStream_t s);
 void free_geometry(DevGeometry *g);
 
-int snapshot_grid(int device, uint32_t n_items, uint32_t cap);
+int snapshot_grid(int device, uint32_t n_items, uint32_t cap, bool pack);  // CTAs for K1 (pack) / K2
 cudaError_t launch_pack(const SnapParams &p, int grid, cudaStream_t s);
 cudaError_t launch_unpack(const SnapParams &p, int grid, cudaStream_t s);
 cudaError_t launch_finalize(const FinalizeParams &p, cudaStream_t s);  // kFinalizeLaunches kernels

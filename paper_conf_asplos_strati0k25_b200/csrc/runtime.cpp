@@ -86,8 +86,9 @@ struct Ckpt {
     bool final_recorded = false;  // ev_final recorded (guarded by mu): finish must not sync it before
     std::atomic<uint32_t> remaining{0};
     cudaEvent_t ev_train = nullptr, ev_begin = nullptr, ev_packed = nullptr, ev_fin_k = nullptr, ev_final = nullptr;
+    cudaEvent_t ev_landed = nullptr;  // copy stream, after the last chunk's D2H (timing)
     double t_call = 0, t_packed = 0, t_landed = 0, t_persisted = 0, t_committed = 0;
-    float pack_ms = 0, fin_ms = 0, k1_busy_ms = 0;
+    float pack_ms = 0, fin_ms = 0, k1_busy_ms = 0, snap_ms = 0;
     // timing events around every K1 launch: the kernel's busy time, without the gaps in which
     // the host waits for ring space between launches (those count in pack_ms, the U-gate span)
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> k1_ev;
@@ -315,6 +316,10 @@ void finish_ckpt(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
     cudaError_t e = cudaEventSynchronize(ck->ev_final);
     if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "finalize"));
     cudaEventElapsedTime(&ck->pack_ms, ck->ev_begin, ck->ev_packed);
+    // K1 start -> last chunk in host memory, on the GPU's clock; Variant A's K1
+    // stores into host memory itself
+    if (c->zerocopy() || c->n == 0 || cudaEventElapsedTime(&ck->snap_ms, ck->ev_begin, ck->ev_landed) != cudaSuccess)
+        ck->snap_ms = ck->pack_ms;
     ck->k1_busy_ms = 0;
     for (auto &p : ck->k1_ev) {
         float ms = 0;
@@ -444,6 +449,7 @@ void orchestrate_loop(pcc_ctx *c) {
                     cudaError_t e = cudaMemcpyAsync(task.dest + o, src + o, len, cudaMemcpyDeviceToHost, c->copy_stream);
                     if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "D2H"));
                 }
+                if (j + task.nchunks == c->n) cudaEventRecord(ck->ev_landed, c->copy_stream);  // before the task
                 task.ev = get_event(c);
                 task.pooled_ev = true;
                 cudaEventRecord(task.ev, c->copy_stream);
@@ -501,6 +507,7 @@ void destroy_ckpt_events(pcc_ctx *c, Ckpt *ck) {
     cudaEventDestroy(ck->ev_train);
     cudaEventDestroy(ck->ev_begin);
     cudaEventDestroy(ck->ev_packed);
+    cudaEventDestroy(ck->ev_landed);
     cudaEventDestroy(ck->ev_fin_k);
     cudaEventDestroy(ck->ev_final);
     for (auto &L : ck->launches) put_event(c, L.ev);
@@ -801,6 +808,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
     cudaEventCreateWithFlags(&ck->ev_train, cudaEventDisableTiming);
     cudaEventCreate(&ck->ev_begin);
     cudaEventCreate(&ck->ev_packed);
+    cudaEventCreate(&ck->ev_landed);
     cudaEventCreate(&ck->ev_fin_k);
     cudaEventCreateWithFlags(&ck->ev_final, cudaEventDisableTiming);
     cudaEventRecord(ck->ev_train, ts);
@@ -832,7 +840,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
         cudaEventRecord(ck->ev_begin, c->pack_stream);
         const auto k1e = k1_events(ck.get());
         cudaEventRecord(k1e.first, c->pack_stream);
-        e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas), c->pack_stream);
+        e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas, true), c->pack_stream);
         cudaEventRecord(k1e.second, c->pack_stream);
         c->launches += c->n ? 1 : 0;
         cudaEvent_t ev = get_event(c);
@@ -871,7 +879,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
             if (done == 0) cudaEventRecord(ck->ev_begin, c->pack_stream);  // K1 time excludes ring waits
             const auto k1e = k1_events(ck.get());
             cudaEventRecord(k1e.first, c->pack_stream);
-            e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas), c->pack_stream);
+            e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas, true), c->pack_stream);
             cudaEventRecord(k1e.second, c->pack_stream);
             c->launches += 1;
             cudaEvent_t ev = get_event(c);
@@ -1047,6 +1055,7 @@ int pcc_info(pcc_ctx *c, pcc_handle h, pcc_ckpt_info *info, uint32_t *crc, uint3
         info->pack_ms = ck->pack_ms;
         info->finalize_ms = ck->fin_ms;
         info->k1_busy_ms = ck->k1_busy_ms;
+        info->snapshot_ms = ck->snap_ms;
         if (crc)
             for (uint32_t i = 0; i < crc_cap && i < ck->crc.size(); ++i) crc[i] = ck->crc[i];
     }
@@ -1209,7 +1218,7 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
         P.first = (uint32_t)j0;
         P.count = (uint32_t)k;
         P.ring_head = whole ? 0 : (R - j0 % R) % R;
-        if ((e = launch_unpack(P, snapshot_grid(c->device, (uint32_t)(k * P.tpc), 0), c->pack_stream)))
+        if ((e = launch_unpack(P, snapshot_grid(c->device, (uint32_t)(k * P.tpc), 0, false), c->pack_stream)))
             rc = cuda_error(e, "K2");
         c->launches += 1;
         cudaEventRecord(ev_k2, c->pack_stream);
@@ -1377,7 +1386,7 @@ int dp_fanout(pcc_ctx *c, uint32_t slot) {
             P.tile_crc = tile;
             P.tables = c->tables;
             P.consts = c->consts;
-            if ((e = launch_unpack(P, snapshot_grid(c->device, (uint32_t)(cnt * P.tpc), 0), c->pack_stream))) {
+            if ((e = launch_unpack(P, snapshot_grid(c->device, (uint32_t)(cnt * P.tpc), 0, false), c->pack_stream))) {
                 rc = cuda_error(e, "fanout K2");
                 break;
             }

@@ -152,3 +152,11 @@ def test_c2_vgg_full_size_parity(pcc):
     o_img, o_crcs, o_dig = _oracle_side(ts, 256, 64 << 20)
     assert np.array_equal(img, o_img)
     assert crcs == o_crcs and dig == o_dig
+
+
+def test_nccl_transport_selftest(pcc):
+    """The library's own NCCL path (nccl_shim.hpp: dlopen, ncclCommInitRank, int64 MIN / MAX
+    allreduce, byte allgather) on a real GPU: one rank, since one GPU cannot host two."""
+    vals = [30, -1, 2**40 + 5, 0, 7]
+    mn, mx, ok = pcc.nccl_selftest(vals)
+    assert mn == vals and mx == vals and ok

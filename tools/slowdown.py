@@ -97,6 +97,7 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
                      staging_bytes=staging_bytes, pack_ctas=pack_ctas, d2h_gbs=d2h_gbs, d2h_quantum=d2h_quantum)
     ck.register(state)
     host_ms = []
+    infos = []  # the checkpoints taken while training runs (contended)
 
     def loop(n, checkpoint, it0):
         handles = []
@@ -122,6 +123,7 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
         total = e0.elapsed_time(e1)
         for h in handles:
             ck.wait(h)
+            infos.append(ck.info(h))
         its = [a.elapsed_time(b) for a, b in per]  # iteration i+1 at index i
         return total, its
 
@@ -159,7 +161,20 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
             "pack_ctas": pack_ctas, "guard": use_guard, "graphs": graphs,
             "d2h_gbs": d2h_gbs or None, "d2h_quantum": d2h_quantum or None, "pace_choice": pace_choice,
             "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
-            "state_bytes": sum(t.numel() * t.element_size() for t in state)}
+            "state_bytes": sum(t.numel() * t.element_size() for t in state),
+            "contended": _contended(infos, sum(t.numel() * t.element_size() for t in state))}
+
+
+def _contended(infos, nbytes):
+    """the snapshot measured while training runs, medians over the checkpoints, on
+    the GPU's clock: K1 alone, the U-gate span, and K1 start -> last chunk landed in host memory
+    (paced when a D2H pace is set)."""
+    if not infos:
+        return None
+    snap = statistics.median(i["snapshot_ms"] for i in infos)
+    return {"checkpoints": len(infos), "k1_busy_ms": statistics.median(i["k1_busy_ms"] for i in infos),
+            "pack_span_ms": statistics.median(i["pack_ms"] for i in infos), "snapshot_ms": snap,
+            "gbs": nbytes / (snap * 1e-3) / 1e9, "bytes": nbytes}
 
 
 def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1, path=None, d2h_gbs=0.0,
@@ -219,6 +234,7 @@ def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1,
                      d2h_gbs=d2h_gbs, d2h_quantum=d2h_quantum)
     ck.register(state)
     geo = ck.geometry()
+    infos = []
 
     def loop(n, checkpoint, it0):
         handles = []
@@ -242,6 +258,7 @@ def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1,
         e1.synchronize()
         for h in handles:
             ck.wait(h)
+            infos.append(ck.info(h))
         return e0.elapsed_time(e1), sorted(a.elapsed_time(b) for a, b in per)
 
     base_t, ck_t, its_b, its_c = [], [], [], []
@@ -267,4 +284,5 @@ def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1,
             "iter_ms_no_ckpt": b / iters, "iter_ms_ckpt": c / iters, "slowdown_pct": (c / b - 1.0) * 100.0,
             "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
             "d2h_gbs": d2h_gbs or None, "d2h_quantum": d2h_quantum or None, "pace_choice": pace_choice,
-            "state_bytes": sum(t.numel() * t.element_size() for t in state)}
+            "state_bytes": sum(t.numel() * t.element_size() for t in state),
+            "contended": _contended(infos, geo["count"] * (64 << 20))}
