@@ -340,10 +340,12 @@ def main():
     ck.register(state)
     geo = ck.geometry()
     slice_bytes = geo["count"] * cb
-    if emu:  # state bytes inside this rank's chunk range (R3: GB/s counts state bytes, not pads)
-        offs, _, _ = pcc.k_layout([(1 << 20, s.nbytes, s.code) for s in specs], 256, cb)
-        lo, hi = geo["first"] * cb, (geo["first"] + geo["count"]) * cb
-        state_bytes = sum(max(0, min(o + s.nbytes, hi) - max(o, lo)) for o, s in zip(offs, specs))
+    # state bytes inside this rank's chunk range (R3: GB/s counts state bytes, not pads)
+    offs, _, _ = pcc.k_layout([(1 << 20, s.nbytes, s.code) for s in specs], 256, cb)
+    lo, hi = geo["first"] * cb, (geo["first"] + geo["count"]) * cb
+    rank_state_bytes = sum(max(0, min(o + s.nbytes, hi) - max(o, lo)) for o, s in zip(offs, specs))
+    if emu:  # one GPU playing one rank: the job is this rank's share
+        state_bytes = rank_state_bytes
     stream = torch.cuda.current_stream()
 
     def barrier():
@@ -460,7 +462,25 @@ def main():
     #                      library configured for training
     #   slowdown_unpaced   eager training, the configuration `value` was measured in
     #   slowdown_graphs    training step as CUDA graphs, tuned pace
+    #   world > 1 (C2): VGG-16 under DDP on every rank, each checkpointing its 1/world slice with
+    #                      the collective commit; the slowdown reported is the max over ranks
     slowdown = slowdown_unpaced = slowdown_graphs = None
+    if world > 1 and not args.no_slowdown and args.config == "c2":
+        from tools.slowdown import vgg16_slowdown
+        ckw = dict(coll) if coll else {"nccl_unique_id": uid}
+        res = {}
+        for name, kw in (("slowdown", dict(d2h_gbs="auto", link_gbs=peak_link)), ("slowdown_unpaced", {})):
+            try:
+                r = vgg16_slowdown(pcc, iters=60, every=10, rank=rank, world=world, ck_kwargs=ckw, **kw)
+                err = 0
+            except Exception as ex:  # noqa: BLE001
+                r, err = {"error": repr(ex)[:300]}, 1
+            t = torch.tensor([r.get("slowdown_pct", 0.0), float(err)], device="cpu" if args.share_gpu else "cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            r["slowdown_pct_rank"] = r.get("slowdown_pct")
+            r["slowdown_pct"] = float(t[0]) if not float(t[1]) else None  # max over ranks
+            res[name] = r
+        slowdown, slowdown_unpaced = res["slowdown"], res["slowdown_unpaced"]
     if rank == 0 and world == 1 and not args.no_slowdown and args.config in ("c2", "c4"):
         try:
             if args.config == "c2":
@@ -505,12 +525,13 @@ def main():
                        else "null sink", "l2": "inputs larger than L2 (state >> 126 MB)"},
             "per_gpu_gbs": value / world,
             "checkpoint_latency_ms_p50": lat_ms,
-            "snapshot_idle": {"ms": idle_ms, "gbs": state_bytes / (idle_ms * 1e-3) / 1e9,
+            "snapshot_idle": {"ms": idle_ms, "gbs": rank_state_bytes / (idle_ms * 1e-3) / 1e9,
                               "def": "K1 start -> last chunk landed in host memory, CUDA events, one checkpoint "
                                      "in flight, median of the warm-up checkpoints after the first"},
             "roofline": {"bound": "hbm", "kernel": "k_snapshot<pack> (K1)", "achieved": k1_achieved,
                          "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": k1_achieved / peaks["hbm_gbs"],
-                         "traffic": load_traffic(f"{args.config}_k1"),
+                         # ncu's DRAM bytes of one W = 1 launch (profiles/k1_traffic.json)
+                         "traffic": load_traffic(f"{args.config}_k1") if world == 1 and not emu else None,
                          "algorithmic_bytes_per_checkpoint": k1_bytes, "k1_ms_per_checkpoint": k1_ms,
                          "k1_launches_per_checkpoint": (launches - 2 * args.steps) / args.steps,  # minus the 2 finalize kernels
                          "pack_span_ms": pack_ms,
@@ -526,7 +547,7 @@ def main():
                     "d2h_bytes_per_step": slice_bytes + 4 * (geo["count"] + 1),
                     # both directions busy every step: the bound is the concurrent H2D + D2H rate
                     "link_peak_bidir_gbs_per_direction": peak_bidir,
-                    "frac_of_bidir": e2e_value / peak_bidir},
+                    "frac_of_bidir": e2e_value / world / peak_bidir},  # per GPU
             "gpu_launches": launches,
             "clocks": clk,
             "slowdown": slowdown,

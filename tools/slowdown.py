@@ -43,17 +43,26 @@ def _auto_pace(pcc, state, chunk_bytes, every, link_gbs, step_fn, stream, rank=0
 
 def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=None, n_inflight=2, flags=None,
                    chunk_bytes=64 << 20, writer_threads=4, staging_bytes=0, pack_ctas=0, use_guard=True,
-                   graphs=False, d2h_gbs=0.0, d2h_quantum=0, link_gbs=None):
+                   graphs=False, d2h_gbs=0.0, d2h_quantum=0, link_gbs=None, rank=0, world=1, ck_kwargs=None):
     """graphs=True: the training step runs as two CUDA graphs (forward + backward, then the
     optimizer step) with the U-gate between them; False: eager PyTorch.  d2h_gbs="auto": the
     tuner's D2H pace (tuner.choose_pace) for `every` x the measured iteration time and the
-    D2H link peak `link_gbs`."""
+    D2H link peak `link_gbs`.
+
+    world > 1 (every rank calls this at the same point, torch.distributed initialised): data
+    parallelism — DistributedDataParallel over the default process group, batch `batch` per rank
+    — and the library at (rank, world): each rank checkpoints its 1/world slice of the replicated
+    state and every checkpoint is followed by the collective commit (allreduce MIN).
+    ck_kwargs: the collectives for PCCheck (allreduce / allgather callbacks or nccl_unique_id)."""
     import torch
     import torchvision
 
     torch.manual_seed(0)
-    dev = torch.device("cuda")
+    dev = torch.device("cuda", torch.cuda.current_device())
     model = torchvision.models.vgg16(weights=None).to(dev)
+    net = model
+    if world > 1:  # DP: gradients allreduced by DDP, parameters / momenta stay replicated
+        net = torch.nn.parallel.DistributedDataParallel(model, device_ids=[dev.index])
     opt = torch.optim.SGD(model.parameters(), lr=1e-3, momentum=0.9)
     x = torch.randn(batch, 3, 224, 224, device=dev)
     y = torch.randint(0, 1000, (batch,), device=dev)
@@ -62,7 +71,7 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
 
     def step():
         opt.zero_grad(set_to_none=True)
-        lossf(model(x), y).backward()
+        lossf(net(x), y).backward()
 
     for _ in range(2):  # momentum buffers exist after the first step
         step()
@@ -79,7 +88,7 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
         g_fb, g_up = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
         opt.zero_grad(set_to_none=True)
         with torch.cuda.graph(g_fb):
-            lossf(model(x), y).backward()
+            lossf(net(x), y).backward()
         with torch.cuda.graph(g_up):
             opt.step()
         step, update = g_fb.replay, g_up.replay
@@ -89,12 +98,13 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
     pace_choice = None
     if d2h_gbs == "auto":  # the tuner's pace for this interval (iteration time measured here)
         d2h_gbs, d2h_quantum, pace_choice = _auto_pace(pcc, state, chunk_bytes, every, link_gbs,
-                                                       lambda: (step(), update()), stream)
+                                                       lambda: (step(), update()), stream, rank, world)
     shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
     path = path or os.path.join(shm, f"pcc_slowdown_{os.getpid()}.pcc")
     ck = pcc.PCCheck(path, chunk_bytes=chunk_bytes, max_inflight=n_inflight,
                      flags=pcc.MAPFILE if flags is None else flags, writer_threads=writer_threads,
-                     staging_bytes=staging_bytes, pack_ctas=pack_ctas, d2h_gbs=d2h_gbs, d2h_quantum=d2h_quantum)
+                     staging_bytes=staging_bytes, pack_ctas=pack_ctas, d2h_gbs=d2h_gbs, d2h_quantum=d2h_quantum,
+                     device=dev.index, rank=rank, world=world, **(ck_kwargs or {}))
     ck.register(state)
     host_ms = []
     infos = []  # the checkpoints taken while training runs (contended)
@@ -113,6 +123,8 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
             if checkpoint and i % every == 0:
                 th = time.perf_counter()
                 handles.append(ck.checkpoint(it0 + i, stream))
+                if world > 1:
+                    ck.commit()  # collective, same program point on every rank
                 host_ms.append((time.perf_counter() - th) * 1e3)
             ev = torch.cuda.Event(enable_timing=True)
             ev.record(stream)
@@ -124,6 +136,8 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
         for h in handles:
             ck.wait(h)
             infos.append(ck.info(h))
+        if world > 1 and handles:
+            ck.commit()
         its = [a.elapsed_time(b) for a, b in per]  # iteration i+1 at index i
         return total, its
 
@@ -150,7 +164,8 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
     b, c = statistics.mean(base_t), statistics.mean(ck_t)
     pct = lambda v, q: sorted(v)[min(len(v) - 1, int(q * len(v)))]  # noqa: E731
     return {"model": "vgg16 fp32 SGD(momentum) batch 32, random init, synthetic inputs"
-                     + (", training step as CUDA graphs" if graphs else ", eager"),
+                     + (", training step as CUDA graphs" if graphs else ", eager")
+                     + (f", DDP over {world} ranks (this rank: {rank}; its 1/{world} slice)" if world > 1 else ""),
             "every": every, "iters": iters, "runs": runs, "N": n_inflight,
             "iter_ms_no_ckpt": b / iters, "iter_ms_ckpt": c / iters,
             "slowdown_pct": (c / b - 1.0) * 100.0,
@@ -162,7 +177,9 @@ def vgg16_slowdown(pcc, iters=60, every=10, warmup=10, batch=32, runs=2, path=No
             "d2h_gbs": d2h_gbs or None, "d2h_quantum": d2h_quantum or None, "pace_choice": pace_choice,
             "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
             "state_bytes": sum(t.numel() * t.element_size() for t in state),
-            "contended": _contended(infos, sum(t.numel() * t.element_size() for t in state))}
+            # this rank's bytes: the whole state at W = 1, its slice (padded chunks) at W > 1
+            "contended": _contended(infos, sum(t.numel() * t.element_size() for t in state) if world == 1
+                                    else _slice_bytes(pcc, state, chunk_bytes, rank, world))}
 
 
 def _contended(infos, nbytes):
