@@ -426,7 +426,11 @@ void orchestrate_loop(pcc_ctx *c) {
                 if (c->mapfile()) {
                     // coalesce chunks of this launch that are contiguous in the ring (and, always,
                     // in the slot) into one copy of up to kCoalesceBytes: fewer, larger D2H
-                    constexpr uint64_t kCoalesceBytes = 64ull << 20;
+                    static const uint64_t kCoalesceBytes = [] {  // PCC_COALESCE_MIB: A/B hook
+                        const char *e = std::getenv("PCC_COALESCE_MIB");
+                        const uint64_t mib = e ? std::strtoull(e, nullptr, 10) : 0;
+                        return (mib ? mib : 64ull) << 20;
+                    }();
                     uint64_t k = 1;
                     const uint64_t kmax = std::max<uint64_t>(1, kCoalesceBytes / c->cb());
                     while (k < kmax && j + k < L.first + L.count && r0 + k < c->ring_slots) ++k;
