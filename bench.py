@@ -451,8 +451,14 @@ def main():
         rdt = time.perf_counter() - t0r
         restore = {"iter": rit, "ms": rdt * 1e3, "gbs": state_bytes / rdt / 1e9, "bad_chunks": len(rbad),
                    "path": "file mapping -> H2D into the HBM ring -> K2 verify+scatter"}
+    barrier()  # W > 1: every GPU probes its link at the same time (the peak at the same concurrency)
     peak_link = d2h_peak_gbs(torch)
     peak_bidir = bidir_peak_gbs(torch)
+    peak_box = peak_link
+    if world > 1:  # the concurrent aggregate of all ranks' D2H peaks (SURVEY §8(d) "box level")
+        tb = torch.tensor([peak_link], device="cpu" if args.share_gpu else "cuda", dtype=torch.float64)
+        dist.all_reduce(tb)
+        peak_box = float(tb.item())
     ck.close()
     if path and os.path.exists(path):
         os.unlink(path)
@@ -538,7 +544,9 @@ def main():
                          "peak_source": "MEASURED_PEAKS.json hbm_gbs (burst copy)"},
             "link_roofline": {"bound": "pcie_d2h", "achieved": link_achieved, "peak": peak_link, "unit": "GB/s",
                               "frac": link_achieved / peak_link,
-                              "peak_source": "pinned 1 GiB cudaMemcpy D2H, measured in this run"},
+                              "peak_source": "pinned 1 GiB cudaMemcpy D2H, measured in this run (all ranks at once)",
+                              "box": {"achieved": value, "peak": peak_box, "frac": value / peak_box,
+                                      "def": "whole-job state GB/s vs the sum of the ranks' concurrent D2H peaks"}},
             "finalize_ms": fin_ms,
             "restore": restore,
             "cpu_baseline": cpu,
