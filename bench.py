@@ -36,6 +36,8 @@ WORKLOADS = {
     "c2": "VGG-16 fp32 params + SGD momentum (1.107 GB), 16 MiB chunks, 2 in-flight checkpoints, DRAM-file target",
     "c3": "OPT-1.3B fp32 params + Adam (15.79 GB), 64 MiB chunks, 4 in-flight checkpoints, DRAM-file target",
     "c4": "BLOOM-7b1 bf16 params + fp32 master + Adam (98.97 GB), 64 MiB chunks, 1/world slice per rank",
+    "bert": "BERT-large QA fp32 params + Adam (PAPER Table 3's 4 GB checkpoint), 64 MiB chunks, 2 in-flight "
+            "checkpoints, DRAM-file target",
 }
 
 
@@ -487,9 +489,16 @@ def main():
             r["slowdown_pct"] = float(t[0]) if not float(t[1]) else None  # max over ranks
             res[name] = r
         slowdown, slowdown_unpaced = res["slowdown"], res["slowdown_unpaced"]
-    if rank == 0 and world == 1 and not args.no_slowdown and args.config in ("c2", "c4"):
+    if rank == 0 and world == 1 and not args.no_slowdown and args.config in ("c2", "c3", "c4", "bert"):
         try:
-            if args.config == "c2":
+            if args.config in ("c3", "bert"):  # the model's own training loop (tools/slowdown.hf_slowdown)
+                del state, host_state
+                torch.cuda.empty_cache()
+                from tools.slowdown import hf_slowdown
+                m = {"c3": "opt13", "bert": "bert"}[args.config]
+                slowdown = hf_slowdown(pcc, m, d2h_gbs="auto", link_gbs=peak_link)
+                slowdown_unpaced = hf_slowdown(pcc, m)
+            elif args.config == "c2":
                 from tools.slowdown import vgg16_slowdown
                 slowdown = vgg16_slowdown(pcc, iters=60, every=10, d2h_gbs="auto", link_gbs=peak_link)
                 slowdown_unpaced = vgg16_slowdown(pcc, iters=60, every=10)

@@ -385,6 +385,28 @@ void persist_loop(pcc_ctx *c) {
 
 void orchestrate_loop(pcc_ctx *c) {
     cudaSetDevice(c->device);
+    // D2H pieces and queue depth (PCC_D2H_PIECE_MIB / PCC_D2H_DEPTH: A/B hooks): 4 x 8 MiB keeps
+    // ~0.6 ms of copies queued — enough to keep the link busy across the host's re-issue latency
+    static const uint64_t d2h_piece = [] {
+        const char *e = std::getenv("PCC_D2H_PIECE_MIB");
+        const uint64_t m = e ? std::strtoull(e, nullptr, 10) : 0;
+        return (m ? m : 8ull) << 20;
+    }();
+    static const size_t d2h_depth = [] {
+        const char *e = std::getenv("PCC_D2H_DEPTH");
+        const size_t d = e ? (size_t)std::strtoull(e, nullptr, 10) : 0;
+        return d ? d : (size_t)4;
+    }();
+    // ... and every d2h_drain pieces the queue runs empty once: a copy engine that always has
+    // work queued from one stream never serves another stream's copy (measured: a 4-byte
+    // .item() on the training stream waited 105 ms for the whole 8 GiB stream at depth 2-4,
+    // 0.1 ms with a gap), and HF models read a flag to the host every forward pass
+    static const uint64_t d2h_drain = [] {
+        const char *e = std::getenv("PCC_D2H_DRAIN");
+        return e ? std::strtoull(e, nullptr, 10) : 8ull;  // 0 = never
+    }();
+    uint64_t since_drain = 0;
+    std::deque<cudaEvent_t> queued;  // completion events of the pieces on the copy engine
     std::shared_ptr<Ckpt> ck;
     while (c->jobs.pop(&ck)) {
         PCC_TRACE("orch: ckpt %llu iter %llu slot %u", (unsigned long long)ck->t.counter,
@@ -443,15 +465,29 @@ void orchestrate_loop(pcc_ctx *c) {
                           (void *)task.dest);
                 const char *src = c->ring + r0 * c->cb();
                 const uint64_t total = task.nchunks * c->cb();
-                const uint64_t q = quantum ? quantum : total;
+                const uint64_t q = quantum ? quantum : std::min<uint64_t>(total, d2h_piece);
                 for (uint64_t o = 0; o < total; o += q) {
                     const uint64_t len = std::min(q, total - o);
                     if (pace) {
                         std::this_thread::sleep_until(t_pace + std::chrono::microseconds(paced_bytes / pace));
                         paced_bytes += len;
                     }
+                    // bounded copy queue with periodic gaps: any D2H the training issues (even a
+                    // 4-byte .item()) waits behind the copies on the copy engine; queued back to
+                    // back, a whole checkpoint (OPT-1.3B: 16 GB) stalled the iteration after each
+                    // checkpoint by ~230 ms
+                    const bool drain = d2h_drain && ++since_drain >= d2h_drain;
+                    if (drain) since_drain = 0;
+                    while (!queued.empty() && (drain || queued.size() >= d2h_depth)) {
+                        cudaEventSynchronize(queued.front());
+                        put_event(c, queued.front());
+                        queued.pop_front();
+                    }
                     cudaError_t e = cudaMemcpyAsync(task.dest + o, src + o, len, cudaMemcpyDeviceToHost, c->copy_stream);
                     if (e != cudaSuccess) fail_ckpt(c, ck, cuda_error(e, "D2H"));
+                    cudaEvent_t qe = get_event(c);
+                    cudaEventRecord(qe, c->copy_stream);
+                    queued.push_back(qe);
                 }
                 if (j + task.nchunks == c->n) cudaEventRecord(ck->ev_landed, c->copy_stream);  // before the task
                 task.ev = get_event(c);
@@ -469,6 +505,10 @@ void orchestrate_loop(pcc_ctx *c) {
         if (!c->zerocopy())
             for (uint32_t j = issued; j < c->n; ++j) ring_release(c, ck->ring_start + j);
         if (c->n == 0 || (unissued && ck->remaining.fetch_sub(unissued) == unissued)) finish_ckpt(c, ck);
+    }
+    for (cudaEvent_t e : queued) {
+        cudaEventSynchronize(e);
+        put_event(c, e);
     }
 }
 

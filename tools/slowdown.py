@@ -303,3 +303,131 @@ def bloom_slowdown(pcc, world=8, iters=40, every=10, warmup=4, seq=2048, runs=1,
             "d2h_gbs": d2h_gbs or None, "d2h_quantum": d2h_quantum or None, "pace_choice": pace_choice,
             "state_bytes": sum(t.numel() * t.element_size() for t in state),
             "contended": _contended(infos, geo["count"] * (64 << 20))}
+
+
+def hf_slowdown(pcc, model="bert", iters=40, every=10, warmup=5, runs=1, path=None, n_inflight=2,
+                chunk_bytes=64 << 20, d2h_gbs=0.0, d2h_quantum=0, link_gbs=None, flags=None, ring_bytes=0,
+                use_guard=True):
+    """The same measurement for two more of north_star's models, random init, synthetic inputs:
+
+    * model="bert": BERT-large with a QA head (BertForQuestionAnswering, 24 layers, hidden 1024),
+      fp32, batch 3 (PAPER Table 3) x 384 tokens (SQuAD's usual length; the paper is
+      silent), Adam(fused) — the "BERT 4 GB" checkpoint of Table 3;
+    * model="opt13": OPT-1.3B (OPTForCausalLM), fp32 params, Adam(fused), bf16
+      autocast, batch 1 (Table 3) x 2048 tokens.
+
+    The checkpointed state is R11's registration of the optimizer (`state_tensors`): param,
+    exp_avg, exp_avg_sq, step per parameter.  Per iteration: forward + backward, pcc_guard (the
+    U-gate of L139), optimizer.step(); every `every`-th iteration, pcc_checkpoint."""
+    import torch
+    torch.manual_seed(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    if model == "bert":
+        from transformers import BertConfig, BertForQuestionAnswering
+        cfg = BertConfig(vocab_size=30522, hidden_size=1024, num_hidden_layers=24, num_attention_heads=16,
+                         intermediate_size=4096, max_position_embeddings=512)
+        net = BertForQuestionAnswering(cfg).to(dev)
+        batch, seq, amp = 3, 384, False
+        ids = torch.randint(0, cfg.vocab_size, (batch, seq), device=dev)
+        starts = torch.randint(0, seq, (batch,), device=dev)
+        ends = torch.randint(0, seq, (batch,), device=dev)
+
+        def fwd_bwd():
+            net(input_ids=ids, start_positions=starts, end_positions=ends).loss.backward()
+        desc = "BERT-large QA fp32, Adam(fused), batch 3 x 384 tokens"
+    elif model == "opt13":
+        from transformers import OPTConfig, OPTForCausalLM
+        cfg = OPTConfig(hidden_size=2048, num_hidden_layers=24, ffn_dim=8192, num_attention_heads=32,
+                        vocab_size=50272, max_position_embeddings=2048, word_embed_proj_dim=2048)
+        net = OPTForCausalLM(cfg).to(dev)
+        batch, seq, amp = 1, 2048, True
+        ids = torch.randint(0, cfg.vocab_size, (batch, seq), device=dev)
+
+        def fwd_bwd():
+            with torch.autocast("cuda", dtype=torch.bfloat16):
+                loss = net(input_ids=ids, labels=ids).loss
+            loss.backward()
+        desc = "OPT-1.3B fp32 params, Adam(fused), bf16 autocast, batch 1 x 2048 tokens"
+    else:
+        raise ValueError(model)
+    net.train()
+    opt = torch.optim.Adam(net.parameters(), lr=1e-5, fused=True)
+    stream = torch.cuda.current_stream()
+
+    def step():
+        opt.zero_grad(set_to_none=True)
+        fwd_bwd()
+
+    for _ in range(2):  # Adam state exists after the first step
+        step()
+        opt.step()
+    state, _ = pcc.state_tensors(opt)
+    pace_choice = None
+    if d2h_gbs == "auto":
+        d2h_gbs, d2h_quantum, pace_choice = _auto_pace(pcc, state, chunk_bytes, every, link_gbs,
+                                                       lambda: (step(), opt.step()), stream)
+    shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
+    path = path or os.path.join(shm, f"pcc_slowdown_{model}_{os.getpid()}.pcc")
+    ck = pcc.PCCheck(None if flags == pcc.NULLSINK else path, chunk_bytes=chunk_bytes, max_inflight=n_inflight,
+                     flags=pcc.MAPFILE if flags is None else flags, ring_bytes=ring_bytes,
+                     staging_bytes=8 * chunk_bytes, d2h_gbs=d2h_gbs, d2h_quantum=d2h_quantum, device=dev.index)
+    ck.register(state)
+    infos = []
+
+    def loop(n, checkpoint, it0):
+        handles = []
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        per = []
+        e0.record(stream)
+        last = e0
+        for i in range(1, n + 1):
+            step()
+            if checkpoint and use_guard:
+                ck.guard(stream)
+            opt.step()
+            if checkpoint and i % every == 0:
+                th = time.perf_counter()
+                handles.append(ck.checkpoint(it0 + i, stream))
+                host_ms.append((time.perf_counter() - th) * 1e3)
+            ev = torch.cuda.Event(enable_timing=True)
+            ev.record(stream)
+            per.append((last, ev))
+            last = ev
+        e1.record(stream)
+        e1.synchronize()
+        for h in handles:
+            ck.wait(h)
+            infos.append(ck.info(h))
+        its = [a.elapsed_time(b) for a, b in per]
+        if checkpoint:
+            by_pos.append(its)
+        return e0.elapsed_time(e1), sorted(its)
+
+    host_ms, by_pos = [], []
+    loop(warmup, False, 0)
+    base_t, ck_t, its_b, its_c = [], [], [], []
+    it0 = 1000
+    for r in range(runs):
+        t, its = loop(iters, False, 0)
+        base_t.append(t)
+        its_b += its
+        t, its = loop(iters, True, it0)
+        it0 += 1000
+        ck_t.append(t)
+        its_c += its
+    ck.drain()
+    ck.close()
+    if os.path.exists(path):
+        os.unlink(path)
+    b, c = statistics.mean(base_t), statistics.mean(ck_t)
+    pct = lambda v, q: sorted(v)[min(len(v) - 1, int(q * len(v)))]  # noqa: E731
+    nbytes = sum(t.numel() * t.element_size() for t in state)
+    return {"model": desc + ", random init, synthetic inputs, eager", "every": every, "iters": iters, "runs": runs,
+            "N": n_inflight, "tensors": len(state), "state_bytes": nbytes,
+            "iter_ms_no_ckpt": b / iters, "iter_ms_ckpt": c / iters, "slowdown_pct": (c / b - 1.0) * 100.0,
+            "p50_ms": [pct(its_b, 0.5), pct(its_c, 0.5)], "p99_ms": [pct(its_b, 0.99), pct(its_c, 0.99)],
+            "d2h_gbs": d2h_gbs or None, "d2h_quantum": d2h_quantum or None, "pace_choice": pace_choice,
+            "host_ckpt_call_ms": statistics.median(host_ms) if host_ms else None,
+            "host_ckpt_call_ms_max": max(host_ms) if host_ms else None,
+            "iter_ms_ckpt_run": by_pos[-1] if by_pos else None,
+            "contended": _contended(infos, nbytes)}
