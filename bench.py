@@ -465,6 +465,16 @@ def main():
     if path and os.path.exists(path):
         os.unlink(path)
 
+    # the oracle as it stands on the host cores, on the same image (before the slowdown runs free
+    # the state)
+    cpu = cpu_all = None
+    if rank == 0 and not args.no_cpu_baseline and args.config in ("c1", "c2", "c3"):
+        from synth import host_bytes
+        hb = [host_bytes(t) for t in state]
+        cpu = cpu_baseline(specs, state, cb, hb=hb)
+        cpu_all = cpu_baseline(specs, state, cb, hb=hb, threads=len(os.sched_getaffinity(0)))
+        del hb
+
     # training slowdown, checkpoint every 10 iterations (BASELINE metric, second half):
     #   slowdown           eager training, D2H paced by the tuner (tuner.choose_pace) — the
     #                      library configured for training
@@ -519,12 +529,6 @@ def main():
         k1_bytes = 2 * slice_bytes  # read the slice's state bytes + write the packed slice (R3: pads count)
         k1_achieved = k1_bytes / (k1_ms * 1e-3) / 1e9
         link_achieved = slice_bytes / (ms_total * 1e-3 / args.steps) / 1e9
-        cpu = cpu_all = None
-        if not args.no_cpu_baseline and args.config in ("c1", "c2", "c3"):
-            from synth import host_bytes
-            hb = [host_bytes(t) for t in state]
-            cpu = cpu_baseline(specs, state, cb, hb=hb)
-            cpu_all = cpu_baseline(specs, state, cb, hb=hb, threads=len(os.sched_getaffinity(0)))
         line = {
             "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_total / args.steps, "higher_is_better": True,

@@ -385,12 +385,11 @@ void persist_loop(pcc_ctx *c) {
 
 void orchestrate_loop(pcc_ctx *c) {
     cudaSetDevice(c->device);
-    // D2H pieces and queue depth (PCC_D2H_PIECE_MIB / PCC_D2H_DEPTH: A/B hooks): 4 x 8 MiB keeps
-    // ~0.6 ms of copies queued — enough to keep the link busy across the host's re-issue latency
+    // D2H pieces and queue depth (PCC_D2H_PIECE_MIB / PCC_D2H_DEPTH: A/B hooks)
     static const uint64_t d2h_piece = [] {
         const char *e = std::getenv("PCC_D2H_PIECE_MIB");
         const uint64_t m = e ? std::strtoull(e, nullptr, 10) : 0;
-        return (m ? m : 8ull) << 20;
+        return (m ? m : 64ull) << 20;
     }();
     static const size_t d2h_depth = [] {
         const char *e = std::getenv("PCC_D2H_DEPTH");
@@ -400,13 +399,21 @@ void orchestrate_loop(pcc_ctx *c) {
     // ... and every d2h_drain pieces the queue runs empty once: a copy engine that always has
     // work queued from one stream never serves another stream's copy (measured: a 4-byte
     // .item() on the training stream waited 105 ms for the whole 8 GiB stream at depth 2-4,
-    // 0.1 ms with a gap), and HF models read a flag to the host every forward pass
+    // 0.1 ms with a gap), and HF models read a flag to the host every forward pass.  2 x 64 MiB
+    // bounds that wait to ~2.4 ms (profiles/r01_d2h_starvation.md: OPT-1.3B unpaced slowdown
+    // 41-46% -> 12.7%, C2 snapshot 55.7 GB/s)
     static const uint64_t d2h_drain = [] {
         const char *e = std::getenv("PCC_D2H_DRAIN");
-        return e ? std::strtoull(e, nullptr, 10) : 8ull;  // 0 = never
+        return e ? std::strtoull(e, nullptr, 10) : 2ull;  // 0 = never
     }();
     uint64_t since_drain = 0;
     std::deque<cudaEvent_t> queued;  // completion events of the pieces on the copy engine
+    // waited for by polling cudaEventQuery between yields: cudaEventSynchronize's spin delayed
+    // the K1 launches of the training thread by ~20 us (K1 0.41 -> 0.43 ms in the C2 bench),
+    // and blocking-sync events wake up too late to keep the link busy (47.6 GB/s)
+    auto q_wait = [](cudaEvent_t e) {
+        while (cudaEventQuery(e) == cudaErrorNotReady) std::this_thread::yield();
+    };
     std::shared_ptr<Ckpt> ck;
     while (c->jobs.pop(&ck)) {
         PCC_TRACE("orch: ckpt %llu iter %llu slot %u", (unsigned long long)ck->t.counter,
@@ -479,7 +486,7 @@ void orchestrate_loop(pcc_ctx *c) {
                     const bool drain = d2h_drain && ++since_drain >= d2h_drain;
                     if (drain) since_drain = 0;
                     while (!queued.empty() && (drain || queued.size() >= d2h_depth)) {
-                        cudaEventSynchronize(queued.front());
+                        q_wait(queued.front());
                         put_event(c, queued.front());
                         queued.pop_front();
                     }

@@ -9,3 +9,4 @@ timeout 600 ncu --set full --clock-control none --import-source on -k regex:k_sn
 timeout 900 python bench.py --config c3 --inflight 4 --steps 6 --no-cpu-baseline > gpurun_out/bench_c3.json 2> gpurun_out/bench_c3.err; echo "bench c3 rc=$?"
 timeout 900 python bench.py --config c4 --emulate-world 8 --steps 6 --no-cpu-baseline > gpurun_out/bench_c4.json 2> gpurun_out/bench_c4.err; echo "bench c4 rc=$?"
 timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err; echo "bench ref rc=$?"
+timeout 900 python bench.py --config bert --steps 10 --no-cpu-baseline > gpurun_out/bench_bert.json 2> gpurun_out/bench_bert.err; echo "bench bert rc=$?"
