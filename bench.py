@@ -107,7 +107,7 @@ def d2h_peak_gbs(torch, nbytes=1 << 30):
     s = torch.cuda.Stream()
     best = 1e9
     with torch.cuda.stream(s):
-        for i in range(5):
+        for i in range(11):
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record(s)
             h.copy_(d, non_blocking=True)

@@ -86,15 +86,16 @@ D2H_QUANTUM = 512 << 10  # bytes per paced copy (0.5 MiB: measured best trade, r
 
 
 def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, margin: float = 0.5,
-                max_margin: float = 0.9, n_inflight: int = 2) -> dict:
+                max_margin: float = 0.5, n_inflight: int = 2) -> dict:
     """D2H pace for training: {"d2h_gbs": G, "d2h_quantum": Q}; G = 0 means unpaced.
 
     The gentlest pace that lands one checkpoint within `margin` of its interval f*t, never below
     half the link (below that the measured cost no longer drops).  When that needs more than
-    the link and N >= 2 checkpoints may overlap (Fig 6), the interval is stretched
-    up to `max_margin` before giving up the pace: a paced copy leaves the link gaps the
-    training's own traffic needs (OPT-1.3B: 15.8 GB every 10 x 44 ms needs 72 GB/s at margin 0.5
-    but 40 GB/s at 0.9)."""
+    the link and N >= 2 checkpoints may overlap (Fig 6), the interval may be
+    stretched up to `max_margin` before giving up the pace.  Off by default (max_margin =
+    margin): measured on OPT-1.3B (15.8 GB every 10 x 44 ms: 72 GB/s at margin 0.5, 40 GB/s at
+    0.9) the stretched pace kept the link busy the whole interval and cost 19.8% against 16.7%
+    unpaced — there the answer is a longer interval (Eq 3's f*), not a pace."""
     if f <= 0 or t <= 0 or link_gbs <= 0:
         raise ValueError("f, t and link_gbs must be positive")
     need = slice_bytes / (margin * f * t) / 1e9  # GB/s to land a checkpoint in margin * f * t

@@ -28,12 +28,13 @@ def test_choose_pace():
     # checkpointing every iteration needs more than the link: unpaced
     assert choose_pace(1_107_296_256, 1, 0.0171, 57.0) == {"d2h_gbs": 0.0, "d2h_quantum": 0,
                                                             "need_gbs": pytest.approx(129.5, rel=1e-3)}
-    # OPT-1.3B (15.8 GB every 10 x 43.8 ms): 72 GB/s at margin 0.5 exceeds the link; with N >= 2
-    # the interval stretches to 0.9 of f*t -> 40 GB/s; with N = 1 it stays unpaced
+    # OPT-1.3B (15.8 GB every 10 x 43.8 ms): 72 GB/s at margin 0.5 exceeds the link -> unpaced by
+    # default; the optional stretch (max_margin 0.9, N >= 2) gives 40 GB/s; never with N = 1
     p = choose_pace(15_789_098_512, 10, 0.0438, 57.0)
-    assert p["need_gbs"] == pytest.approx(72.1, rel=1e-2)
+    assert p["need_gbs"] == pytest.approx(72.1, rel=1e-2) and p["d2h_gbs"] == 0.0
+    p = choose_pace(15_789_098_512, 10, 0.0438, 57.0, max_margin=0.9)
     assert p["d2h_gbs"] == pytest.approx(15_789_098_512 / (0.9 * 10 * 0.0438) / 1e9) and p["d2h_quantum"] == D2H_QUANTUM
-    assert choose_pace(15_789_098_512, 10, 0.0438, 57.0, n_inflight=1)["d2h_gbs"] == 0.0
+    assert choose_pace(15_789_098_512, 10, 0.0438, 57.0, max_margin=0.9, n_inflight=1)["d2h_gbs"] == 0.0
     with pytest.raises(ValueError):
         choose_pace(1, 0, 1.0, 1.0)
 
