@@ -479,7 +479,7 @@ def main():
     #   slowdown           eager training, D2H paced by the tuner (tuner.choose_pace) — the
     #                      library configured for training
     #   slowdown_unpaced   eager training, the configuration `value` was measured in
-    #   slowdown_graphs    training step as CUDA graphs, tuned pace
+    #   slowdown_graphs    training step as CUDA graphs (VGG-16: tuned pace; OPT-1.3B: unpaced, host <= 2 replays ahead)
     #   world > 1 (C2): VGG-16 under DDP on every rank, each checkpointing its 1/world slice with
     #                      the collective commit; the slowdown reported is the max over ranks
     slowdown = slowdown_unpaced = slowdown_graphs = None
@@ -508,6 +508,10 @@ def main():
                 m = {"c3": "opt13", "bert": "bert"}[args.config]
                 slowdown = hf_slowdown(pcc, m, d2h_gbs="auto", link_gbs=peak_link)
                 slowdown_unpaced = hf_slowdown(pcc, m)
+                if m == "opt13":  # the step as one CUDA graph: immune to the eager launch penalty
+                    from tools.opt_graph_slowdown import opt13_graph_slowdown
+                    torch.cuda.empty_cache()
+                    slowdown_graphs = opt13_graph_slowdown()
             elif args.config == "c2":
                 from tools.slowdown import vgg16_slowdown
                 slowdown = vgg16_slowdown(pcc, iters=60, every=10, d2h_gbs="auto", link_gbs=peak_link)

@@ -12,70 +12,71 @@ import torch  # noqa: E402
 import paper_conf_asplos_strati0k25_b200 as pcc  # noqa: E402
 from transformers import OPTConfig, OPTForCausalLM  # noqa: E402
 
-dev = torch.device("cuda", 0)
-attn = sys.argv[1] if len(sys.argv) > 1 else "sdpa"
-host_lead = int(sys.argv[2]) if len(sys.argv) > 2 else 0  # >0: host waits for replay i-lead before enqueuing i
-cfg = OPTConfig(hidden_size=2048, num_hidden_layers=24, ffn_dim=8192, num_attention_heads=32, vocab_size=50272,
-                max_position_embeddings=2048, word_embed_proj_dim=2048)
-cfg._attn_implementation = attn
-net = OPTForCausalLM(cfg).to(dev).train()
-ids = torch.randint(0, cfg.vocab_size, (1, 2048), device=dev)
-mask = torch.ones(1, 2048, dtype=torch.long, device=dev)
-opt = torch.optim.Adam(net.parameters(), lr=1e-5, fused=True, capturable=True)
+def opt13_graph_slowdown(attn="sdpa", host_lead=2, iters=40, every=10):
+    """Returns the result dict printed by the script (see the module docstring)."""
+    dev = torch.device("cuda", 0)
+    cfg = OPTConfig(hidden_size=2048, num_hidden_layers=24, ffn_dim=8192, num_attention_heads=32, vocab_size=50272,
+                    max_position_embeddings=2048, word_embed_proj_dim=2048)
+    cfg._attn_implementation = attn
+    net = OPTForCausalLM(cfg).to(dev).train()
+    ids = torch.randint(0, cfg.vocab_size, (1, 2048), device=dev)
+    mask = torch.ones(1, 2048, dtype=torch.long, device=dev)
+    opt = torch.optim.Adam(net.parameters(), lr=1e-5, fused=True, capturable=True)
 
+    def step():
+        opt.zero_grad(set_to_none=False)
+        with torch.autocast("cuda", dtype=torch.bfloat16, cache_enabled=False):
+            loss = net(input_ids=ids, attention_mask=mask, labels=ids).loss
+        loss.backward()
+        opt.step()
 
-def step():
-    opt.zero_grad(set_to_none=False)
-    with torch.autocast("cuda", dtype=torch.bfloat16, cache_enabled=False):
-        loss = net(input_ids=ids, attention_mask=mask, labels=ids).loss
-    loss.backward()
-    opt.step()
-
-
-side = torch.cuda.Stream()
-side.wait_stream(torch.cuda.current_stream())
-with torch.cuda.stream(side):
-    for _ in range(3):
+    side = torch.cuda.Stream()
+    side.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(side):
+        for _ in range(3):
+            step()
+    torch.cuda.current_stream().wait_stream(side)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
         step()
-torch.cuda.current_stream().wait_stream(side)
-g = torch.cuda.CUDAGraph()
-with torch.cuda.graph(g):
-    step()
-stream = torch.cuda.current_stream()
-state, _ = pcc.state_tensors(opt)
-path = f"/dev/shm/pcc_optgraph_{os.getpid()}.pcc"
-ck = pcc.PCCheck(path, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.MAPFILE, staging_bytes=8 * (64 << 20), device=0)
-ck.register(state)
+    stream = torch.cuda.current_stream()
+    state, _ = pcc.state_tensors(opt)
+    path = f"/dev/shm/pcc_optgraph_{os.getpid()}.pcc"
+    ck = pcc.PCCheck(path, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.MAPFILE, staging_bytes=8 * (64 << 20), device=0)
+    ck.register(state)
+
+    def loop(n, checkpoint, it0):
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
+        evs[0].record(stream)
+        hs = []
+        for i in range(1, n + 1):
+            if checkpoint and i % every == 1 and i > 1:
+                ck.guard(stream)
+            if host_lead and i > host_lead:
+                evs[i - host_lead].synchronize()
+            g.replay()
+            if checkpoint and i % every == 0:
+                hs.append(ck.checkpoint(it0 + i, stream))
+            evs[i].record(stream)
+        evs[-1].synchronize()
+        for h in hs:
+            ck.wait(h)
+        return [evs[i - 1].elapsed_time(evs[i]) for i in range(1, n + 1)]
+
+    loop(5, False, 0)
+    loop(12, True, 100)
+    base = loop(iters, False, 0)
+    withck = loop(iters, True, 1000)
+    ck.drain()
+    ck.close()
+    os.unlink(path)
+    mb, mc = sum(base) / len(base), sum(withck) / len(withck)
+    return ({"model": f"OPT-1.3B, whole step as one CUDA graph ({attn} attention)", "every": every,
+                      "iter_ms_no_ckpt": mb, "iter_ms_ckpt": mc, "slowdown_pct": 100 * (mc / mb - 1),
+                      "iters_ms_ckpt": [round(x, 1) for x in withck], "host_lead": host_lead,
+                      "state_bytes": sum(t.numel() * t.element_size() for t in state), "tensors": len(state)})
 
 
-def loop(n, checkpoint, it0):
-    evs = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
-    evs[0].record(stream)
-    hs = []
-    for i in range(1, n + 1):
-        if checkpoint and i % 10 == 1 and i > 1:
-            ck.guard(stream)
-        if host_lead and i > host_lead:
-            evs[i - host_lead].synchronize()
-        g.replay()
-        if checkpoint and i % 10 == 0:
-            hs.append(ck.checkpoint(it0 + i, stream))
-        evs[i].record(stream)
-    evs[-1].synchronize()
-    for h in hs:
-        ck.wait(h)
-    return [evs[i - 1].elapsed_time(evs[i]) for i in range(1, n + 1)]
-
-
-loop(5, False, 0)
-loop(12, True, 100)
-base = loop(40, False, 0)
-withck = loop(40, True, 1000)
-ck.drain()
-ck.close()
-os.unlink(path)
-mb, mc = sum(base) / len(base), sum(withck) / len(withck)
-print(json.dumps({"model": f"OPT-1.3B, whole step as one CUDA graph ({attn} attention)", "every": 10,
-                  "iter_ms_no_ckpt": mb, "iter_ms_ckpt": mc, "slowdown_pct": 100 * (mc / mb - 1),
-                  "iters_ms_ckpt": [round(x, 1) for x in withck], "host_lead": host_lead,
-                  "state_bytes": sum(t.numel() * t.element_size() for t in state), "tensors": len(state)}))
+if __name__ == "__main__":
+    print(json.dumps(opt13_graph_slowdown(sys.argv[1] if len(sys.argv) > 1 else "sdpa",
+                                          int(sys.argv[2]) if len(sys.argv) > 2 else 2)))
