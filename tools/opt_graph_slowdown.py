@@ -6,6 +6,7 @@ follows a checkpoint (conservative: the whole step waits for K1, not only the op
 import json
 import os
 import sys
+import time
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
@@ -56,16 +57,20 @@ def opt13_graph_slowdown(attn="sdpa", host_lead=2, iters=40, every=10):
                 evs[i - host_lead].synchronize()
             g.replay()
             if checkpoint and i % every == 0:
+                th = time.perf_counter()
                 hs.append(ck.checkpoint(it0 + i, stream))
+                host_ms.append(round((time.perf_counter() - th) * 1e3, 2))
             evs[i].record(stream)
         evs[-1].synchronize()
         for h in hs:
             ck.wait(h)
         return [evs[i - 1].elapsed_time(evs[i]) for i in range(1, n + 1)]
 
+    host_ms = []
     loop(5, False, 0)
     loop(12, True, 100)
     base = loop(iters, False, 0)
+    host_ms.clear()
     withck = loop(iters, True, 1000)
     ck.drain()
     ck.close()
@@ -73,7 +78,7 @@ def opt13_graph_slowdown(attn="sdpa", host_lead=2, iters=40, every=10):
     mb, mc = sum(base) / len(base), sum(withck) / len(withck)
     return ({"model": f"OPT-1.3B, whole step as one CUDA graph ({attn} attention)", "every": every,
                       "iter_ms_no_ckpt": mb, "iter_ms_ckpt": mc, "slowdown_pct": 100 * (mc / mb - 1),
-                      "iters_ms_ckpt": [round(x, 1) for x in withck], "host_lead": host_lead,
+                      "iters_ms_ckpt": [round(x, 1) for x in withck], "host_lead": host_lead, "host_ckpt_call_ms": host_ms,
                       "state_bytes": sum(t.numel() * t.element_size() for t in state), "tensors": len(state)})
 
 
