@@ -13,7 +13,7 @@ import torch  # noqa: E402
 import paper_conf_asplos_strati0k25_b200 as pcc  # noqa: E402
 from transformers import OPTConfig, OPTForCausalLM  # noqa: E402
 
-def opt13_graph_slowdown(attn="sdpa", host_lead=2, iters=40, every=10):
+def opt13_graph_slowdown(attn="sdpa", host_lead=2, iters=40, every=10, ring_slices=1):
     """Returns the result dict printed by the script (see the module docstring)."""
     dev = torch.device("cuda", 0)
     cfg = OPTConfig(hidden_size=2048, num_hidden_layers=24, ffn_dim=8192, num_attention_heads=32, vocab_size=50272,
@@ -43,7 +43,8 @@ def opt13_graph_slowdown(attn="sdpa", host_lead=2, iters=40, every=10):
     stream = torch.cuda.current_stream()
     state, _ = pcc.state_tensors(opt)
     path = f"/dev/shm/pcc_optgraph_{os.getpid()}.pcc"
-    ck = pcc.PCCheck(path, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.MAPFILE, staging_bytes=8 * (64 << 20), device=0)
+    ck = pcc.PCCheck(path, chunk_bytes=64 << 20, max_inflight=2, flags=pcc.MAPFILE, staging_bytes=8 * (64 << 20), device=0,
+                     ring_bytes=0 if ring_slices == 1 else ring_slices * (-(-sum(t.numel() * t.element_size() for t in state) // (64 << 20))) * (64 << 20))
     ck.register(state)
 
     def loop(n, checkpoint, it0):
@@ -78,10 +79,11 @@ def opt13_graph_slowdown(attn="sdpa", host_lead=2, iters=40, every=10):
     mb, mc = sum(base) / len(base), sum(withck) / len(withck)
     return ({"model": f"OPT-1.3B, whole step as one CUDA graph ({attn} attention)", "every": every,
                       "iter_ms_no_ckpt": mb, "iter_ms_ckpt": mc, "slowdown_pct": 100 * (mc / mb - 1),
-                      "iters_ms_ckpt": [round(x, 1) for x in withck], "host_lead": host_lead, "host_ckpt_call_ms": host_ms,
+                      "iters_ms_ckpt": [round(x, 1) for x in withck], "host_lead": host_lead, "ring_slices": ring_slices, "host_ckpt_call_ms": host_ms,
                       "state_bytes": sum(t.numel() * t.element_size() for t in state), "tensors": len(state)})
 
 
 if __name__ == "__main__":
     print(json.dumps(opt13_graph_slowdown(sys.argv[1] if len(sys.argv) > 1 else "sdpa",
-                                          int(sys.argv[2]) if len(sys.argv) > 2 else 2)))
+                                          int(sys.argv[2]) if len(sys.argv) > 2 else 2,
+                                          ring_slices=int(sys.argv[3]) if len(sys.argv) > 3 else 1)))
