@@ -42,6 +42,8 @@ def lib():
         u8p, u32p, u64p = C.POINTER(C.c_uint8), C.POINTER(C.c_uint32), C.POINTER(C.c_uint64)
         _lib.orc_crc32c.restype = C.c_uint32
         _lib.orc_crc32c.argtypes = [C.c_void_p, C.c_uint64]
+        _lib.orc_crc32c_extend.restype = C.c_uint32
+        _lib.orc_crc32c_extend.argtypes = [C.c_uint32, C.c_void_p, C.c_uint64]
         _lib.orc_layout.argtypes = [C.c_uint32, u64p, C.c_uint32, C.c_uint64, u64p, u64p, u64p]
         _lib.orc_slice.argtypes = [C.c_uint64, C.c_uint32, C.c_uint32, u64p, u64p]
         _lib.orc_pack.argtypes = [C.c_uint32, C.POINTER(C.c_void_p), u64p, u64p, C.c_uint64, C.c_uint64,
@@ -94,6 +96,13 @@ def crc32c(data) -> int:
     return int(lib().orc_crc32c(b.ctypes.data, b.nbytes))
 
 
+def crc32c_extend(crc, data) -> int:
+    """O3/O4 resumed: CRC32C(A || data) given crc = CRC32C(A) (crc = 0 for an empty A),
+    byte at a time — the slice digest of a multi-GB image in one pass, chunk by chunk."""
+    b = np.ascontiguousarray(data).view(np.uint8)
+    return int(lib().orc_crc32c_extend(crc, b.ctypes.data, b.nbytes))
+
+
 def layout(nbytes, align=256, chunk_bytes=4 << 20):
     """O1: image offsets, end and chunk count C (R1-R3; PAPER L127/L281 'contiguous')."""
     nb, nbp = _u64(nbytes)
@@ -140,6 +149,30 @@ def pack_chunks_sparse(all_nbytes, srcs_by_index, align, chunk_bytes, first_chun
     offa, offp = _u64([off[i] for i in idx])
     out = np.empty(count * chunk_bytes, dtype=np.uint8)
     lib().orc_pack(len(idx), ptrs, nbp, offp, chunk_bytes, first_chunk, count, out.ctypes.data)
+    return out
+
+
+def pack_range(all_nbytes, fetch, align, chunk_bytes, first_chunk, count):
+    """O2 for image bytes [lo, hi) = [first_chunk*CB, (first_chunk+count)*CB), written with
+    numpy slice copies instead of the C byte loop (which walks every byte of every tensor it
+    is handed, far too slow to cover a 16-32 GB image chunk by chunk):
+
+        image[max(off_i, lo) - lo : min(off_i + n_i, hi) - lo]
+            = tensor_i[max(lo - off_i, 0) : min(hi - off_i, n_i)]     for every tensor i,
+
+    zero everywhere else (R1, R3; "contiguous").  ``fetch(i, a, b)`` returns
+    bytes [a, b) of tensor i as a uint8 array.  Pinned against ``pack`` (the C byte loop) by
+    brute force in tests/test_oracle.py."""
+    off, end, c = layout(all_nbytes, align, chunk_bytes)
+    lo, hi = first_chunk * chunk_bytes, (first_chunk + count) * chunk_bytes
+    out = np.zeros(hi - lo, dtype=np.uint8)
+    for i, n in enumerate(all_nbytes):
+        o = int(off[i])
+        a, b = max(o, lo), min(o + int(n), hi)
+        if b > a:
+            piece = np.asarray(fetch(i, a - o, b - o), dtype=np.uint8).reshape(-1)
+            assert piece.nbytes == b - a, f"fetch({i}) returned {piece.nbytes} bytes, wanted {b - a}"
+            out[a - lo:b - lo] = piece
     return out
 
 

@@ -60,6 +60,13 @@ ORC_EXPORT uint32_t orc_crc32c(const uint8_t *p, uint64_t n) {
     return orc_crc_update(0xFFFFFFFFu, p, n) ^ 0xFFFFFFFFu;
 }
 
+/* CRC32C(A || B) from crc = CRC32C(A): undo the xorout, keep feeding bytes one at a time,
+ * apply the xorout again.  The same byte loop as orc_crc32c, resumable, so a slice digest
+ * (O4) of a multi-GB image can be computed in one pass over chunks handed in order. */
+ORC_EXPORT uint32_t orc_crc32c_extend(uint32_t crc, const uint8_t *p, uint64_t n) {
+    return orc_crc_update(crc ^ 0xFFFFFFFFu, p, n) ^ 0xFFFFFFFFu;
+}
+
 /* ------------------------------------------------------------------ O1 layout */
 /* Tensors in registration order; off_0 = 0; off_i = align_up(off_{i-1} + nbytes_{i-1}, align);
  * end = off_last + nbytes_last; C = ceil(end / chunk_bytes).  (R1, R2, R3) */

@@ -147,6 +147,73 @@ def test_slices_partition_chunks(world):
         assert seen == list(range(c))
 
 
+def test_slices_hand_values():
+    """orc_slice against hand-computed floor(r*C/W) bounds (FORMAT.md "Image"); a
+    remainder-first split (the first C % W ranks take one extra chunk) would give (0,9)/(9,8)
+    for C=17, W=2 and (0,3)/(3,3)/(6,2)/(8,2) for C=10, W=4, so it fails here."""
+    assert [oracle.rank_slice(17, r, 2) for r in range(2)] == [(0, 8), (8, 9)]
+    assert [oracle.rank_slice(10, r, 4) for r in range(4)] == [(0, 2), (2, 3), (5, 2), (7, 3)]
+    # C4 (BLOOM-7b1, 1475 chunks of 64 MiB) at W = 8: floor(1475 r / 8) = 0, 184, 368, 553, 737, 921, 1106, 1290
+    assert [oracle.rank_slice(1475, r, 8) for r in range(8)] == [
+        (0, 184), (184, 184), (368, 185), (553, 184), (737, 184), (921, 185), (1106, 184), (1290, 185)]
+    assert oracle.rank_slice(3, 2, 4) == (1, 1) and oracle.rank_slice(3, 0, 4) == (0, 0)
+
+
+def test_slot_geometry_hand_values():
+    """orc_header_bytes / orc_slot_stride / orc_slot_offset against FORMAT.md "File", by hand:
+    H = align_up(96 + 4n + 4, 4096), stride = align_up(H + n*CB, 4096), slot s at 8192 + s*stride."""
+    MiB = 1 << 20
+    # n = 17, CB = 4 MiB: H = 4096 (168 B of fields); stride = 4096 + 71,303,168 = 71,307,264
+    assert oracle.header_bytes(17) == 4096
+    assert oracle.slot_stride(17, 4 * MiB) == 71_307_264
+    assert oracle.slot_offset(0, 17, 4 * MiB) == 8192
+    assert oracle.slot_offset(2, 17, 4 * MiB) == 8192 + 2 * 71_307_264 == 142_622_720
+    # n = 999 still fits one page (96 + 3996 + 4 = 4096); n = 1000 needs two (4100 -> 8192)
+    assert oracle.header_bytes(999) == 4096 and oracle.header_bytes(1000) == 8192
+    # n = 1000, CB = 48 (not page-aligned data): stride = align_up(8192 + 48,000, 4096) = 57,344
+    assert oracle.slot_stride(1000, 48) == 57_344
+    assert oracle.slot_offset(3, 1000, 48) == 8192 + 3 * 57_344 == 180_224
+    # n = 0: a bare header page per slot
+    assert oracle.slot_stride(0, 64 * MiB) == 4096 and oracle.slot_offset(5, 0, 64 * MiB) == 8192 + 5 * 4096
+    # C3 (OPT-1.3B, 236 chunks of 64 MiB): H = align_up(96 + 944 + 4, 4096) = 4096
+    assert oracle.slot_offset(4, 236, 64 * MiB) == 8192 + 4 * (4096 + 236 * 64 * MiB)
+
+
+def test_crc32c_extend_is_crc_of_concatenation(hwcrc):
+    rng = np.random.default_rng(11)
+    for na, nb in [(0, 0), (0, 7), (1, 1), (5, 4096), (4096, 3), (1 << 16, 1 << 16)]:
+        a = rng.integers(0, 256, na, dtype=np.uint8)
+        b = rng.integers(0, 256, nb, dtype=np.uint8)
+        ab = np.concatenate([a, b])
+        assert oracle.crc32c_extend(oracle.crc32c(a), b) == hwcrc(ab) == oracle.crc32c(ab)
+    assert oracle.crc32c_extend(0, b"123456789") == 0xE3069283  # RFC 3720 check value from an empty prefix
+
+
+def test_pack_range_equals_byte_loop():
+    """pack_range (numpy slices) == pack (the C byte loop) on every chunk range of tiny
+    registrations and on chunk ranges of C1 (97 tensors, 10 under 16 B, one spanning 8 chunks)."""
+    rng = np.random.default_rng(12)
+    sizes = [0, 1, 15, 16, 17, 40]
+    for combo in itertools.product(sizes, repeat=3):
+        srcs = [rng.integers(1, 256, n, dtype=np.uint8) for n in combo]
+        for cb, align in ((16, 16), (48, 256), (64, 16)):
+            full = oracle.pack(srcs, align=align, chunk_bytes=cb)
+            c = full.nbytes // cb
+            for first in range(c):
+                for cnt in range(1, c - first + 1):
+                    got = oracle.pack_range(list(combo), lambda i, a, b: srcs[i][a:b], align, cb, first, cnt)
+                    assert got.tobytes() == full[first * cb:(first + cnt) * cb].tobytes()
+    from synth import config_tensors
+    specs = config_tensors("c1")
+    nb = [s.nbytes for s in specs]
+    srcs = [rng.integers(0, 256, n, dtype=np.uint8) for n in nb]
+    cb = 4 << 20
+    full = oracle.pack(srcs, 256, cb)
+    for first, cnt in [(0, 1), (3, 5), (16, 1), (0, 17)]:
+        got = oracle.pack_range(nb, lambda i, a, b: srcs[i][a:b], 256, cb, first, cnt)
+        assert np.array_equal(got, full[first * cb:(first + cnt) * cb])
+
+
 # -------------------------------------------------- P5 on-file records, parsed independently
 def test_slot_header_independent_parse(hwcrc):
     crcs = [0x11111111, 0xDEADBEEF, 0x0]
@@ -344,3 +411,32 @@ def test_pack_chunks_sparse_equals_full_pack():
                 if sizes[i] and int(off[i]) < (j + 1) * cb and int(off[i]) + sizes[i] > j * cb}
         part = oracle.pack_chunks_sparse(sizes, need, 256, cb, j, 1)
         assert part.tobytes() == full[j * cb:(j + 1) * cb].tobytes()
+
+
+def test_fullsize_checker_accepts_oracle_file_and_rejects_faults(tmp_path):
+    """The full-size GPU parity helper (tests/test_fullsize_gpu.oracle_check_slot) on a file the
+    oracle wrote: it must accept it, and name a changed data byte, a changed CRC-table entry and a
+    changed digest."""
+    from synth import config_tensors, make_state, host_bytes
+    from test_fullsize_gpu import oracle_check_slot
+    specs = config_tensors("c1")
+    ts = make_state(specs, "cpu", seed=3, it=1)
+    cb = 4 << 20
+    p = str(tmp_path / "c1.pcc")
+    oracle.write_checkpoint(p, [host_bytes(t) for t in ts], [s.code for s in specs], 256, cb, 0, 1, 2, 1, 5, 1, 1)
+    n = oracle.layout([s.nbytes for s in specs], 256, cb)[2]
+    assert oracle_check_slot(p, specs, ts, 1, n, 0, cb)[0] == n
+    base = oracle.slot_offset(1, n, cb)
+    H = oracle.header_bytes(n)
+    for at, what in [(base + H + 3 * cb + 12345, "chunks differ"), (base + 96 + 4 * 5, "header CRC32C"),
+                     (base + 72, "digest")]:
+        with open(p, "r+b") as f:
+            f.seek(at)
+            b = f.read(1)
+            f.seek(at)
+            f.write(bytes([b[0] ^ 0x10]))
+        with pytest.raises(AssertionError, match=what):
+            oracle_check_slot(p, specs, ts, 1, n, 0, cb)
+        with open(p, "r+b") as f:
+            f.seek(at)
+            f.write(b)
