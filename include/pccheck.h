@@ -175,15 +175,20 @@ PCC_API int pcc_register(pcc_ctx *ctx, const pcc_tensor *t, uint32_t n);
 
 /* Starts checkpoint `iter` of the registered state as it is on `train_stream` now.
  * Listing 1 lines 3-11 (sample the pointer, take the counter, dequeue a free slot — this
- * BLOCKS while N checkpoints hold all slots, the paper's stall), then launches K1 on the
- * library's pack stream after an event on train_stream.  Returns once every K1 launch of
- * the checkpoint is enqueued (it may block for HBM ring space when ring_bytes < slice).
- * iter must strictly increase (-PCC_EORDER).  *out receives the handle. */
+ * BLOCKS while N checkpoints hold all N+1 slots, the paper's stall, L139 Fig 6), records an
+ * event on train_stream and hands the checkpoint to the library's threads: the packer launches
+ * K1 on the pack stream after that event (in windows, as HBM ring space frees), the
+ * orchestrator streams the chunks to host memory.  It never waits for ring space or for an
+ * earlier checkpoint's transfer.  iter must strictly increase (-PCC_EORDER).  *out receives
+ * the handle.  World > 1: COLLECTIVE when a rank has no free slot (backpressure rounds). */
 PCC_API int pcc_checkpoint(pcc_ctx *ctx, uint64_t iter, void *train_stream, pcc_handle *out);
 
-/* U-gate (L139): makes train_stream wait (cudaStreamWaitEvent) until the newest
- * checkpoint's K1 finished reading the registered tensors.  Call before the optimizer step
- * that overwrites them.  No-op when nothing is packing. */
+/* U-gate (L139): makes train_stream wait until the newest checkpoint's K1 finished reading
+ * the registered tensors.  Call before the optimizer step that overwrites them.  The wait is
+ * on the GPU (cuStreamWaitValue32 on a word the pack stream writes after the checkpoint's
+ * last K1 window): the call returns at once even if K1 has not been launched yet.  Without
+ * stream memory operations (or with PCC_NO_STREAM_MEMOPS set) the host waits until the K1
+ * windows are enqueued, then the stream waits for their event.  No-op before any checkpoint. */
 PCC_API int pcc_guard(pcc_ctx *ctx, void *train_stream);
 
 PCC_API int pcc_poll(pcc_ctx *ctx, pcc_handle h, int *state);

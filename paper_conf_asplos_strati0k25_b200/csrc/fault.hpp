@@ -7,6 +7,7 @@
 //   header       before a COMPLETE slot header is written
 //   pointer      before a pointer record is written
 //   mid_pointer  after writing the first half of a pointer record
+//   k1_fail      (not a crash) the n-th K1 window launch reports a launch failure
 #pragma once
 #include <csignal>
 #include <cstdlib>

@@ -14,6 +14,7 @@
 // Chunks of a checkpoint land contiguously in their slot (L127, L281: "contiguous on
 // storage"), N checkpoints may be in flight (L139, Fig 6), copy and persist overlap per
 // chunk (L141, Fig 7).
+#include <cuda.h>  // driver-API types for the stream memory operations (fetched via cudart, no -lcuda)
 #include <cuda_runtime.h>
 #include <fcntl.h>
 #include <sys/mman.h>
@@ -31,6 +32,7 @@
 #include <map>
 #include <memory>
 #include <mutex>
+#include <set>
 #include <string>
 #include <thread>
 #include <vector>
@@ -42,6 +44,7 @@
 #include "kernels.hpp"
 #include "layout.hpp"
 #include "nccl_shim.hpp"
+#include "nvtx3/nvToolsExt.h"
 
 namespace pcc {
 
@@ -53,6 +56,43 @@ int cuda_error(cudaError_t e, const char *what) {
 }
 
 using Clock = std::chrono::steady_clock;
+
+// NVTX ranges around the pipeline stages (pack, D2H, persist, commit): free when no tool is
+// attached; nsys / ncu --nvtx show them on the timeline (SURVEY §8(d) "Evidence").
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange &) = delete;
+    NvtxRange &operator=(const NvtxRange &) = delete;
+};
+
+// Stream memory operations (cuStreamWaitValue32 / cuStreamWriteValue32), fetched from the
+// driver through cudart so the library needs no -lcuda.  The U-gate uses them: the training
+// stream waits ON THE GPU for a word the pack stream writes after a checkpoint's last K1 window,
+// so pcc_checkpoint / pcc_guard never block the calling thread on ring space.
+using WaitValue32Fn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+using WriteValue32Fn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+struct StreamMemOps {
+    WaitValue32Fn wait32 = nullptr;
+    WriteValue32Fn write32 = nullptr;
+    bool ok() const { return wait32 && write32; }
+};
+static const StreamMemOps &stream_mem_ops() {
+    static const StreamMemOps ops = [] {
+        StreamMemOps o;
+        if (std::getenv("PCC_NO_STREAM_MEMOPS")) return o;  // test hook: the host-blocking fallback
+        cudaDriverEntryPointQueryResult q1 = cudaDriverEntryPointSymbolNotFound, q2 = q1;
+        void *w = nullptr, *x = nullptr;
+        if (cudaGetDriverEntryPointByVersion("cuStreamWaitValue32", &w, 12000, cudaEnableDefault, &q1) == cudaSuccess &&
+            cudaGetDriverEntryPointByVersion("cuStreamWriteValue32", &x, 12000, cudaEnableDefault, &q2) == cudaSuccess &&
+            q1 == cudaDriverEntryPointSuccess && q2 == cudaDriverEntryPointSuccess) {
+            o.wait32 = reinterpret_cast<WaitValue32Fn>(w);
+            o.write32 = reinterpret_cast<WriteValue32Fn>(x);
+        }
+        return o;
+    }();
+    return ops;
+}
 
 // PCC_TRACE=1: one stderr line per pipeline event (debugging hangs on the GPU box)
 static bool trace_on() {
@@ -75,8 +115,10 @@ struct Launch {
 
 struct Ckpt {
     Ticket t;
+    uint32_t seq = 0;  // 1, 2, ... in pcc_checkpoint order: the U-gate word value after its last K1
     std::atomic<int> state{PCC_ST_QUEUED};
     std::atomic<int> err{0};
+    std::atomic<bool> packed_recorded{false};  // ev_packed recorded by the packer thread
     uint64_t ring_start = 0;
     std::mutex mu;
     std::condition_variable cv;
@@ -172,12 +214,23 @@ struct pcc_ctx {
     std::vector<uint32_t *> crc_host;  // pinned [n + 1] (+ digest)
     uint32_t *rexpect_dev = nullptr, *rbad_dev = nullptr;  // restore: expected CRCs, bad flags [n]
 
-    // HBM ring (Variant B)
+    // HBM ring (Variant B).  Positions are absolute (checkpoint k's chunk j sits at position
+    // ring_start(k) + j, in ring slot position % ring_slots); [ring_tail, ring_head) are
+    // reserved, a position is released once its D2H landed (or it was never issued), and the
+    // tail only advances over released positions — keyed by absolute position, so a release
+    // can never alias a slot another in-flight chunk still owns.
     char *ring = nullptr;
     uint64_t ring_slots = 0, ring_head = 0, ring_tail = 0;
-    std::vector<uint8_t> ring_done;
+    std::set<uint64_t> ring_released;  // released positions >= ring_tail
     std::mutex ring_mu;
     std::condition_variable ring_cv;
+
+    // U-gate: device word written (stream-ordered) after each checkpoint's last K1 window
+    uint32_t *gate_dev = nullptr;
+    uint32_t issued_seq = 0;                 // caller thread: seq of the newest pcc_checkpoint
+    std::atomic<uint32_t> packed_seq{0};     // packer: seq whose K1 windows + gate write are enqueued
+    std::mutex pk_mu;
+    std::condition_variable pk_cv;
 
     // pinned staging pool (PWRITE / NULLSINK)
     char *staging = nullptr;
@@ -198,7 +251,9 @@ struct pcc_ctx {
     std::condition_variable ck_cv;
     std::map<uint64_t, std::shared_ptr<Ckpt>> ckpts;  // handle (= counter) -> record
 
-    // threads
+    // threads: packer (K1 windows, in checkpoint order), orchestrator (D2H), persist pool
+    BlockingQueue<std::shared_ptr<Ckpt>> packs;
+    std::thread packer;
     BlockingQueue<std::shared_ptr<Ckpt>> jobs;
     BlockingQueue<PersistTask> tasks;
     std::thread orchestrator;
@@ -257,12 +312,13 @@ void set_state(pcc_ctx *c, Ckpt *ck, int st) {
     c->ck_cv.notify_all();
 }
 
-void ring_release(pcc_ctx *c, uint64_t idx) {
+void ring_release(pcc_ctx *c, uint64_t pos) {
     {
         std::lock_guard<std::mutex> lk(c->ring_mu);
-        c->ring_done[idx % c->ring_slots] = 1;
-        while (c->ring_tail < c->ring_head && c->ring_done[c->ring_tail % c->ring_slots]) {
-            c->ring_done[c->ring_tail % c->ring_slots] = 0;
+        if (pos >= c->ring_tail) c->ring_released.insert(pos);
+        auto it = c->ring_released.begin();
+        while (it != c->ring_released.end() && *it == c->ring_tail) {
+            it = c->ring_released.erase(it);
             ++c->ring_tail;
         }
     }
@@ -342,6 +398,7 @@ void finish_ckpt(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
         return;
     }
     set_state(c, ck.get(), PCC_ST_PERSISTED);
+    NvtxRange nv("pcc.commit");
     int st = PCC_ST_FAILED;
     int rc = c->engine->complete(ck->t, ck->crc.data(), ck->digest, &st);
     PCC_TRACE("finish: ckpt %llu committed state %d rc %d", (unsigned long long)ck->t.counter, st, rc);
@@ -357,6 +414,7 @@ void persist_loop(pcc_ctx *c) {
     cudaSetDevice(c->device);
     PersistTask task;
     while (c->tasks.pop(&task)) {
+        NvtxRange nv("pcc.persist");
         Ckpt *ck = task.ck.get();
         PCC_TRACE("persist: ckpt %llu chunk %u wait", (unsigned long long)ck->t.counter, task.j);
         cudaError_t e = cudaEventSynchronize(task.ev);
@@ -396,15 +454,18 @@ void orchestrate_loop(pcc_ctx *c) {
         const size_t d = e ? (size_t)std::strtoull(e, nullptr, 10) : 0;
         return d ? d : (size_t)4;
     }();
-    // ... and every d2h_drain pieces the queue runs empty once: a copy engine that always has
+    // ... and every d2h_drain BYTES the queue runs empty once: a copy engine that always has
     // work queued from one stream never serves another stream's copy (measured: a 4-byte
     // .item() on the training stream waited 105 ms for the whole 8 GiB stream at depth 2-4,
-    // 0.1 ms with a gap), and HF models read a flag to the host every forward pass.  2 x 64 MiB
+    // 0.1 ms with a gap), and HF models read a flag to the host every forward pass.  128 MiB
     // bounds that wait to ~2.4 ms (profiles/r01_d2h_starvation.md: OPT-1.3B unpaced slowdown
-    // 41-46% -> 12.7%, C2 snapshot 55.7 GB/s)
+    // 41-46% -> 12.7%, C2 snapshot 55.7 GB/s).  Counted in bytes, not copies: with the pacer's
+    // 0.5 MiB quanta a per-copy count drained every 1 MiB and the host round trips capped the
+    // paced transfer at ~9.5 GB/s against a 28.6 GB/s target.  A paced transfer
+    // never drains: its own gaps already let other streams' copies through.
     static const uint64_t d2h_drain = [] {
-        const char *e = std::getenv("PCC_D2H_DRAIN");
-        return e ? std::strtoull(e, nullptr, 10) : 2ull;  // 0 = never
+        const char *e = std::getenv("PCC_D2H_DRAIN_MIB");
+        return (e ? std::strtoull(e, nullptr, 10) : 128ull) << 20;  // 0 = never
     }();
     uint64_t since_drain = 0;
     std::deque<cudaEvent_t> queued;  // completion events of the pieces on the copy engine
@@ -418,10 +479,8 @@ void orchestrate_loop(pcc_ctx *c) {
     while (c->jobs.pop(&ck)) {
         PCC_TRACE("orch: ckpt %llu iter %llu slot %u", (unsigned long long)ck->t.counter,
                   (unsigned long long)ck->t.iter, ck->t.slot);
-        if (c->fd >= 0) {
-            int rc = c->engine->filling(ck->t);  // R18: before any data byte of this slot changes
-            if (rc) fail_ckpt(c, ck, rc);
-        }
+        NvtxRange nv("pcc.d2h");
+        // (the FILLING header of R18 was written by the packer before its first K1 launch)
         size_t li = 0;
         uint32_t issued = 0;
         // D2H pacing (pcc_config d2h_mbps / d2h_quantum): copies of at most `quantum` bytes,
@@ -483,8 +542,9 @@ void orchestrate_loop(pcc_ctx *c) {
                     // 4-byte .item()) waits behind the copies on the copy engine; queued back to
                     // back, a whole checkpoint (OPT-1.3B: 16 GB) stalled the iteration after each
                     // checkpoint by ~230 ms
-                    const bool drain = d2h_drain && ++since_drain >= d2h_drain;
+                    const bool drain = !pace && d2h_drain && since_drain >= d2h_drain;
                     if (drain) since_drain = 0;
+                    since_drain += len;
                     while (!queued.empty() && (drain || queued.size() >= d2h_depth)) {
                         q_wait(queued.front());
                         put_event(c, queued.front());
@@ -604,6 +664,145 @@ bool any_inflight(pcc_ctx *c) {
     return false;
 }
 
+// The packer thread: K1 for one checkpoint, after the caller's event on the training stream.
+// Runs checkpoints strictly in pcc_checkpoint order, so K1 windows, the U-gate word and the
+// finalize kernels are stream-ordered on the pack stream.  Waiting for HBM ring space
+// (Variant B with a ring smaller than the slices in flight) happens HERE, not in the caller:
+// the training thread only enqueues, and the U-gate holds the training
+// stream on the GPU instead (pcc_guard).
+void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
+    NvtxRange nv("pcc.pack");
+    const uint32_t s = ck->t.slot;
+    cudaStreamWaitEvent(c->pack_stream, ck->ev_train, 0);
+    if (c->fd >= 0) {
+        // R18: the reused slot's header becomes FILLING before any data byte of the slot changes
+        // — before K1 is even launched, which matters in ZEROCOPY mode where K1 stores straight
+        // into the slot's file pages
+        int rc = c->engine->filling(ck->t);
+        if (rc) fail_ckpt(c, ck, rc);
+    }
+    set_state(c, ck.get(), PCC_ST_PACKING);
+    SnapParams P{};
+    P.rows = c->rows_dev;
+    P.row_begin = c->row_begin_dev;
+    P.tile_rows = c->tile_rows_dev;
+    P.chunk_bytes = c->cb();
+    P.tpc = c->geom.tpc;
+    P.tile_crc = c->tile_crc_dev[s];
+    P.tables = c->tables;
+    P.consts = c->consts;
+    cudaError_t e = cudaSuccess;
+    // publishes a successful window to the orchestrator (a failed one never is)
+    auto publish = [&](uint32_t first, uint32_t count) {
+        cudaEvent_t ev = get_event(c);
+        cudaEventRecord(ev, c->pack_stream);
+        {
+            std::lock_guard<std::mutex> lk(ck->mu);
+            ck->launches.push_back({first, count, ev});
+            ck->launched = first + count;
+        }
+        ck->cv.notify_all();  // the orchestrator may already be waiting for this launch
+    };
+    cudaEventRecord(ck->ev_begin, c->pack_stream);  // K1 time excludes the caller's wait
+    if (c->zerocopy()) {  // Variant A: K1 stores into the registered file mapping over PCIe
+        P.first = 0;
+        P.count = (uint32_t)c->n;
+        P.ring_base = c->map_dev + c->slot_data_off(s);
+        P.ring_head = 0;
+        P.ring_slots = c->n ? c->n : 1;
+        const auto k1e = k1_events(ck.get());
+        cudaEventRecord(k1e.first, c->pack_stream);
+        e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas, true), c->pack_stream);
+        cudaEventRecord(k1e.second, c->pack_stream);
+        c->launches += c->n ? 1 : 0;
+        if (e == cudaSuccess) publish(0, (uint32_t)c->n);
+    } else {  // Variant B: HBM ring, windowed by ring space
+        {
+            std::lock_guard<std::mutex> lk(c->ring_mu);
+            ck->ring_start = c->ring_head;
+            c->ring_head += c->n;
+        }
+        uint64_t done = 0;
+        while (done < c->n && e == cudaSuccess) {
+            uint64_t k;
+            {
+                // launch windows of at least a quarter ring (or the rest of the slice): when the
+                // link is the bottleneck the ring frees a chunk or two at a time, and a K1 launch
+                // per freed chunk pays the table load and launch latency each time (C3 with
+                // N = 4 over a 2-slice ring: 114 launches per checkpoint, 11.7 ms of K1 instead
+                // of 5.7).  The chunks already packed keep the copy engine busy meanwhile.
+                const uint64_t want = std::min<uint64_t>(c->n - done, std::max<uint64_t>(1, c->ring_slots / 4));
+                std::unique_lock<std::mutex> lk(c->ring_mu);
+                c->ring_cv.wait(lk, [&] { return c->ring_tail + c->ring_slots >= ck->ring_start + done + want; });
+                k = std::min<uint64_t>(c->n - done, c->ring_tail + c->ring_slots - (ck->ring_start + done));
+            }
+            P.first = (uint32_t)done;
+            P.count = (uint32_t)k;
+            P.ring_base = c->ring;
+            P.ring_head = ck->ring_start % c->ring_slots;
+            P.ring_slots = c->ring_slots;
+            const auto k1e = k1_events(ck.get());
+            cudaEventRecord(k1e.first, c->pack_stream);
+            // PCC_FAULT=k1_fail:<n>: the n-th K1 window of the process fails to launch (test hook)
+            e = fault_hit("k1_fail") ? cudaErrorLaunchFailure
+                                     : launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas, true),
+                                                   c->pack_stream);
+            cudaEventRecord(k1e.second, c->pack_stream);
+            c->launches += 1;
+            if (e != cudaSuccess) break;
+            publish((uint32_t)done, (uint32_t)k);
+            done += k;
+        }
+    }
+    cudaEventRecord(ck->ev_packed, c->pack_stream);
+    ck->packed_recorded = true;
+    // open the U-gate: stream-ordered after the last K1 window (written even when a launch
+    // failed, so a guarded training stream is never left waiting)
+    if (stream_mem_ops().ok())
+        stream_mem_ops().write32(reinterpret_cast<CUstream>(c->pack_stream), reinterpret_cast<CUdeviceptr>(c->gate_dev),
+                                 ck->seq, CU_STREAM_WRITE_VALUE_DEFAULT);
+    cudaEventRecord(c->ev_guard, c->pack_stream);
+    {
+        std::lock_guard<std::mutex> lk(c->pk_mu);
+        c->packed_seq.store(ck->seq);
+    }
+    c->pk_cv.notify_all();
+    // chunk CRCs -> slice digest, then the table to pinned host memory for the header
+    cudaMemsetAsync(c->scratch_dev[s], 0, 4 * sizeof(uint32_t), c->pack_stream);
+    FinalizeParams F{};
+    F.tile_crc = c->tile_crc_dev[s];
+    F.tables = c->tables;
+    F.n = (uint32_t)c->n;
+    F.tpc = c->geom.tpc;
+    F.tile_shift = c->geom.tile_shift;
+    F.chunk_shift = c->geom.chunk_shift;
+    F.ff = c->geom.ff;
+    F.crc_out = c->crc_dev[s];
+    F.scratch = c->scratch_dev[s];
+    if (e == cudaSuccess) e = launch_finalize(F, c->pack_stream);
+    cudaEventRecord(ck->ev_fin_k, c->pack_stream);
+    if (c->n) c->launches += kFinalizeLaunches;
+    cudaMemcpyAsync(c->crc_dev[s] + c->n, c->scratch_dev[s] + 3, 4, cudaMemcpyDeviceToDevice, c->pack_stream);
+    cudaMemcpyAsync(c->crc_host[s], c->crc_dev[s], (c->n + 1) * sizeof(uint32_t), cudaMemcpyDeviceToHost,
+                    c->pack_stream);
+    cudaEventRecord(ck->ev_final, c->pack_stream);
+    {
+        std::lock_guard<std::mutex> lk(ck->mu);
+        ck->final_recorded = true;
+        if (e != cudaSuccess) {
+            fail_ckpt(c, ck, cuda_error(e, "K1 launch"));
+            ck->launch_failed = true;
+        }
+    }
+    ck->cv.notify_all();
+}
+
+void pack_loop(pcc_ctx *c) {
+    cudaSetDevice(c->device);
+    std::shared_ptr<Ckpt> ck;
+    while (c->packs.pop(&ck)) pack_one(c, ck);
+}
+
 }  // namespace
 
 // ============================================================================ C ABI
@@ -674,6 +873,8 @@ int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
     cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking);
     cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking);
     cudaEventCreateWithFlags(&c->ev_guard, cudaEventDisableTiming);
+    if ((e = cudaMalloc(&c->gate_dev, sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "U-gate word");
+    if ((e = cudaMemset(c->gate_dev, 0, sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "U-gate word");
     if (!nullsink) {
         int flags = O_RDWR | O_CREAT;
         if ((cfg->flags & PCC_ODIRECT) && !(cfg->flags & PCC_MAPFILE)) flags |= O_DIRECT;
@@ -692,6 +893,7 @@ int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
         cudaMallocHost(&c->red_host, 4 * sizeof(int64_t));
     }
     pcc_ctx *raw = c.get();
+    raw->packer = std::thread(pack_loop, raw);
     raw->orchestrator = std::thread(orchestrate_loop, raw);
     for (uint32_t i = 0; i < raw->cfg.writer_threads; ++i) raw->persisters.emplace_back(persist_loop, raw);
     *out = c.release();
@@ -773,7 +975,7 @@ int pcc_register(pcc_ctx *c, const pcc_tensor *t, uint32_t nt) {
         if (r > 8 * nn) r = 8 * nn;  // more than 8 slices of ring cannot be used (N in flight)
         c->ring_slots = r;
         if ((e = cudaMalloc(&c->ring, r * c->cb())) != cudaSuccess) return cuda_error(e, "HBM ring");
-        c->ring_done.assign(r, 0);
+        c->ring_released.clear();
         c->ring_head = c->ring_tail = 0;
     }
     // staging pool (c = M / b, L176)
@@ -855,127 +1057,30 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
         c->engine->wait_free(-1);  // the stall of L139 / Fig 6 when N checkpoints are in flight
     }
     cudaSetDevice(c->device);
-    const uint32_t s = ck->t.slot;
     cudaEventCreateWithFlags(&ck->ev_train, cudaEventDisableTiming);
     cudaEventCreate(&ck->ev_begin);
     cudaEventCreate(&ck->ev_packed);
     cudaEventCreate(&ck->ev_landed);
     cudaEventCreate(&ck->ev_fin_k);
     cudaEventCreateWithFlags(&ck->ev_final, cudaEventDisableTiming);
-    cudaEventRecord(ck->ev_train, ts);
-    cudaStreamWaitEvent(c->pack_stream, ck->ev_train, 0);
+    // the state as it is on the training stream now: K1 starts after this event
+    cudaError_t e = cudaEventRecord(ck->ev_train, ts);
+    if (e != cudaSuccess) {
+        c->engine->fail(ck->t);
+        destroy_ckpt_events(c, ck.get());
+        return cuda_error(e, "event on the training stream");
+    }
     ck->remaining = (uint32_t)c->n;
+    ck->seq = ++c->issued_seq;
     {
         std::lock_guard<std::mutex> lk(c->ck_mu);
         c->ckpts[ck->t.counter] = ck;
     }
-    ck->state = PCC_ST_PACKING;
-    c->jobs.push(ck);  // the orchestrator follows the launches as they are published
-
-    SnapParams P{};
-    P.rows = c->rows_dev;
-    P.row_begin = c->row_begin_dev;
-    P.tile_rows = c->tile_rows_dev;
-    P.chunk_bytes = c->cb();
-    P.tpc = c->geom.tpc;
-    P.tile_crc = c->tile_crc_dev[s];
-    P.tables = c->tables;
-    P.consts = c->consts;
-    cudaError_t e = cudaSuccess;
-    if (c->zerocopy()) {  // Variant A: K1 stores into the registered file mapping over PCIe
-        P.first = 0;
-        P.count = (uint32_t)c->n;
-        P.ring_base = c->map_dev + c->slot_data_off(s);
-        P.ring_head = 0;
-        P.ring_slots = c->n ? c->n : 1;
-        cudaEventRecord(ck->ev_begin, c->pack_stream);
-        const auto k1e = k1_events(ck.get());
-        cudaEventRecord(k1e.first, c->pack_stream);
-        e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas, true), c->pack_stream);
-        cudaEventRecord(k1e.second, c->pack_stream);
-        c->launches += c->n ? 1 : 0;
-        cudaEvent_t ev = get_event(c);
-        cudaEventRecord(ev, c->pack_stream);
-        {
-            std::lock_guard<std::mutex> lk(ck->mu);
-            ck->launches.push_back({0, (uint32_t)c->n, ev});
-            ck->launched = (uint32_t)c->n;
-        }
-        ck->cv.notify_all();  // the orchestrator may already be waiting for this launch
-    } else {  // Variant B: HBM ring, windowed by ring space
-        {
-            std::lock_guard<std::mutex> lk(c->ring_mu);
-            ck->ring_start = c->ring_head;
-            c->ring_head += c->n;
-        }
-        uint64_t done = 0;
-        while (done < c->n && e == cudaSuccess) {
-            uint64_t k;
-            {
-                // launch windows of at least a quarter ring (or the rest of the slice): when the
-                // link is the bottleneck the ring frees a chunk or two at a time, and a K1 launch
-                // per freed chunk pays the table load and launch latency each time (C3 with
-                // N = 4 over a 2-slice ring: 114 launches per checkpoint, 11.7 ms of K1 instead
-                // of 5.7).  The chunks already packed keep the copy engine busy meanwhile.
-                const uint64_t want = std::min<uint64_t>(c->n - done, std::max<uint64_t>(1, c->ring_slots / 4));
-                std::unique_lock<std::mutex> lk(c->ring_mu);
-                c->ring_cv.wait(lk, [&] { return c->ring_tail + c->ring_slots >= ck->ring_start + done + want; });
-                k = std::min<uint64_t>(c->n - done, c->ring_tail + c->ring_slots - (ck->ring_start + done));
-            }
-            P.first = (uint32_t)done;
-            P.count = (uint32_t)k;
-            P.ring_base = c->ring;
-            P.ring_head = ck->ring_start % c->ring_slots;
-            P.ring_slots = c->ring_slots;
-            if (done == 0) cudaEventRecord(ck->ev_begin, c->pack_stream);  // K1 time excludes ring waits
-            const auto k1e = k1_events(ck.get());
-            cudaEventRecord(k1e.first, c->pack_stream);
-            e = launch_pack(P, snapshot_grid(c->device, P.count * P.tpc, c->cfg.pack_ctas, true), c->pack_stream);
-            cudaEventRecord(k1e.second, c->pack_stream);
-            c->launches += 1;
-            cudaEvent_t ev = get_event(c);
-            cudaEventRecord(ev, c->pack_stream);
-            {
-                std::lock_guard<std::mutex> lk(ck->mu);
-                ck->launches.push_back({(uint32_t)done, (uint32_t)k, ev});
-                ck->launched = (uint32_t)(done + k);
-            }
-            ck->cv.notify_all();
-            done += k;
-        }
-    }
-    if (c->n == 0) cudaEventRecord(ck->ev_begin, c->pack_stream);
-    cudaEventRecord(ck->ev_packed, c->pack_stream);
-    cudaEventRecord(c->ev_guard, c->pack_stream);
     c->guard_armed = true;
-    // chunk CRCs -> slice digest, then the table to pinned host memory for the header
-    cudaMemsetAsync(c->scratch_dev[s], 0, 4 * sizeof(uint32_t), c->pack_stream);
-    FinalizeParams F{};
-    F.tile_crc = c->tile_crc_dev[s];
-    F.tables = c->tables;
-    F.n = (uint32_t)c->n;
-    F.tpc = c->geom.tpc;
-    F.tile_shift = c->geom.tile_shift;
-    F.chunk_shift = c->geom.chunk_shift;
-    F.ff = c->geom.ff;
-    F.crc_out = c->crc_dev[s];
-    F.scratch = c->scratch_dev[s];
-    if (e == cudaSuccess) e = launch_finalize(F, c->pack_stream);
-    cudaEventRecord(ck->ev_fin_k, c->pack_stream);
-    if (c->n) c->launches += kFinalizeLaunches;
-    cudaMemcpyAsync(c->crc_dev[s] + c->n, c->scratch_dev[s] + 3, 4, cudaMemcpyDeviceToDevice, c->pack_stream);
-    cudaMemcpyAsync(c->crc_host[s], c->crc_dev[s], (c->n + 1) * sizeof(uint32_t), cudaMemcpyDeviceToHost,
-                    c->pack_stream);
-    cudaEventRecord(ck->ev_final, c->pack_stream);
-    {
-        std::lock_guard<std::mutex> lk(ck->mu);
-        ck->final_recorded = true;
-        if (e != cudaSuccess) {
-            fail_ckpt(c, ck, cuda_error(e, "K1 launch"));
-            ck->launch_failed = true;
-        }
-    }
-    ck->cv.notify_all();
+    // K1 (packer thread) and the D2H (orchestrator) follow asynchronously; this call never
+    // waits for ring space or for the previous checkpoint's transfer
+    c->jobs.push(ck);
+    c->packs.push(ck);
     *out = ck->t.counter;
     return PCC_OK;
 }
@@ -983,7 +1088,23 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
 int pcc_guard(pcc_ctx *c, void *train_stream) {
     if (!c) return set_error(PCC_EINVAL, "ctx");
     if (!c->guard_armed) return PCC_OK;
-    cudaError_t e = cudaStreamWaitEvent(static_cast<cudaStream_t>(train_stream), c->ev_guard, 0);
+    cudaStream_t ts = static_cast<cudaStream_t>(train_stream);
+    const uint32_t want = c->issued_seq;
+    if (stream_mem_ops().ok()) {
+        // the training stream waits on the GPU until the pack stream wrote `want` — after the
+        // newest checkpoint's last K1 window, whenever the packer gets to launch it
+        CUresult r = stream_mem_ops().wait32(reinterpret_cast<CUstream>(ts), reinterpret_cast<CUdeviceptr>(c->gate_dev),
+                                             want, CU_STREAM_WAIT_VALUE_GEQ);
+        if (r != CUDA_SUCCESS) return set_error(PCC_ECUDA, "cuStreamWaitValue32 (U-gate)");
+        return PCC_OK;
+    }
+    // fallback without stream memory operations: the host waits until the packer enqueued the
+    // newest checkpoint's K1 windows, then the stream waits for their event (still exact)
+    {
+        std::unique_lock<std::mutex> lk(c->pk_mu);
+        c->pk_cv.wait(lk, [&] { return (int32_t)(c->packed_seq.load() - want) >= 0; });
+    }
+    cudaError_t e = cudaStreamWaitEvent(ts, c->ev_guard, 0);
     return e == cudaSuccess ? PCC_OK : cuda_error(e, "guard");
 }
 
@@ -1002,7 +1123,8 @@ int pcc_poll(pcc_ctx *c, pcc_handle h, int *state) {
     auto ck = find_ck(c, h);
     if (!ck) return set_error(PCC_EINVAL, "unknown handle");
     int s = ck->state.load();
-    if (s == PCC_ST_PACKING && cudaEventQuery(ck->ev_packed) == cudaSuccess) s = PCC_ST_PACKED;
+    if (s == PCC_ST_PACKING && ck->packed_recorded.load() && cudaEventQuery(ck->ev_packed) == cudaSuccess)
+        s = PCC_ST_PACKED;
     if (s == PCC_ST_LOCAL_COMMIT && c->cfg.world > 1) {
         uint64_t g = c->engine->global_iter();
         if (g != UINT64_MAX && g >= ck->t.iter) s = PCC_ST_GLOBAL_COMMIT;
@@ -1150,6 +1272,8 @@ int pcc_latest(const char *path, uint64_t *global_iter, uint64_t *local_iter) {
 int pcc_close(pcc_ctx *c) {
     if (!c) return PCC_OK;
     pcc_drain(c, -1);
+    c->packs.close();
+    if (c->packer.joinable()) c->packer.join();
     c->jobs.close();
     if (c->orchestrator.joinable()) c->orchestrator.join();
     c->tasks.close();
@@ -1165,6 +1289,7 @@ int pcc_close(pcc_ctx *c) {
     free_registration(c);
     for (auto e : c->evpool) cudaEventDestroy(e);
     cudaEventDestroy(c->ev_guard);
+    if (c->gate_dev) cudaFree(c->gate_dev);
     cudaStreamDestroy(c->pack_stream);
     cudaStreamDestroy(c->copy_stream);
     cudaStreamDestroy(c->aux_stream);

@@ -243,3 +243,120 @@ def test_edge_cases(pcc, shm):
         with pytest.raises(pcc.PCCError) as ei:
             ck.restore()
         assert ei.value.code in (pcc.ELAYOUT, pcc.ENOENT)
+
+
+def _expected_images(specs, seed, iters, cb):
+    """The oracle image of the state perturb_state(seed, it) produces, per iter (filled on a
+    separate set of device tensors, so nothing here waits on the library's streams)."""
+    out = {}
+    ref = make_state(specs, "cuda", seed=seed, it=0)
+    for it in iters:
+        perturb_state(ref, specs, seed=seed, it=it)
+        out[it] = oracle.pack([host_bytes(t) for t in ref], 256, cb)
+    return out
+
+
+@pytest.mark.parametrize("memops", [True, False])
+def test_small_ring_caller_never_blocks_and_gate_exact(pcc, shm, memops):
+    """Variant B with a 3-chunk HBM ring for a 17-chunk slice and a slow (paced) transfer: K1
+    windows wait for ring space in the packer thread, so pcc_checkpoint + pcc_guard return at
+    once, while the U-gate still holds the training stream on the GPU: the state
+    is rewritten right after each guard with NO host synchronisation, and every checkpoint must
+    still hold the state of its own call (L139).  memops=False runs the host-side fallback."""
+    import subprocess
+    import sys
+    import json
+    code = f"""
+import json, os, sys, time
+sys.path.insert(0, {os.path.dirname(os.path.dirname(os.path.abspath(__file__)))!r})
+import torch, oracle
+import paper_conf_asplos_strati0k25_b200 as pcc
+from synth import config_tensors, make_state, perturb_state, host_bytes
+sys.path.insert(0, os.path.join({os.path.dirname(os.path.dirname(os.path.abspath(__file__)))!r}, 'tests'))
+from test_runtime_gpu import _expected_images
+specs = config_tensors('c1'); cb = 4 << 20; iters = list(range(10, 70, 10))
+exp = _expected_images(specs, 4, iters, cb)
+ts = make_state(specs, 'cuda', seed=4, it=0)
+calls = []
+with pcc.PCCheck({shm!r}, chunk_bytes=cb, max_inflight=len(iters) + 1, flags=pcc.MAPFILE, ring_bytes=3 * cb,
+                 d2h_gbs=1.0, d2h_quantum=1 << 20) as ck:
+    ck.register(ts)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    hs = []
+    for it in iters:
+        perturb_state(ts, specs, seed=4, it=it)   # the 'update' of iteration it (stream-ordered)
+        a = time.perf_counter(); hs.append(ck.checkpoint(it)); ck.guard(); calls.append(time.perf_counter() - a)
+    issued = time.perf_counter() - t0
+    perturb_state(ts, specs, seed=4, it=999)      # rewritten after the last guard too
+    for h in hs:
+        ck.wait(h)
+    total = time.perf_counter() - t0
+    ok = []
+    for h in hs:
+        inf = ck.info(h, with_crc=True)
+        ok.append(inf['state_name'] == 'LOCAL_COMMIT' and inf['crc'] == [int(x) for x in oracle.chunk_crcs(exp[inf['iter']], cb)]
+                  and inf['digest'] == oracle.crc32c(exp[inf['iter']]))
+print(json.dumps({{'calls_ms': [c * 1e3 for c in calls], 'issued_s': issued, 'total_s': total, 'ok': ok}}))
+"""
+    env = dict(os.environ)
+    if not memops:
+        env["PCC_NO_STREAM_MEMOPS"] = "1"
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=600, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    res = json.loads(r.stdout.strip().splitlines()[-1])
+    assert all(res["ok"]), res
+    # 6 checkpoints x 71 MB at a 1 GB/s pace take >= 0.4 s; the caller spent almost none of it
+    assert res["total_s"] > 0.35, res
+    if memops:
+        assert max(res["calls_ms"]) < 20 and res["issued_s"] < 0.25 * res["total_s"], res
+
+
+def test_failed_k1_window_frees_ring_and_later_checkpoints_match(pcc, shm):
+    """a K1 window that fails to launch (PCC_FAULT=k1_fail:3, N=2, a 5-chunk ring
+    for a 17-chunk slice) fails ITS checkpoint (pointer untouched) without publishing the
+    window, gives its ring positions back only in order, and the next checkpoints are the
+    oracle's images byte for byte (no chunk of theirs is overwritten before its D2H)."""
+    import subprocess
+    import sys
+    import json
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = f"""
+import json, os, sys
+sys.path.insert(0, {root!r}); sys.path.insert(0, os.path.join({root!r}, 'tests'))
+import torch, oracle
+import paper_conf_asplos_strati0k25_b200 as pcc
+from synth import config_tensors, make_state, perturb_state
+from test_runtime_gpu import _expected_images
+specs = config_tensors('c1'); cb = 4 << 20; iters = [10, 20, 30, 40]
+exp = _expected_images(specs, 6, iters, cb)
+ts = make_state(specs, 'cuda', seed=6, it=0)
+out = {{}}
+with pcc.PCCheck({shm!r}, chunk_bytes=cb, max_inflight=2, flags=pcc.MAPFILE, ring_bytes=5 * cb) as ck:
+    ck.register(ts)
+    for it in iters:
+        perturb_state(ts, specs, seed=6, it=it)
+        h = ck.checkpoint(it); ck.guard()
+        try:
+            ck.wait(h)
+        except pcc.PCCError as e:
+            pass
+        inf = ck.info(h, with_crc=True)
+        good = inf['state_name'] == 'LOCAL_COMMIT' and inf['crc'] == [int(x) for x in oracle.chunk_crcs(exp[it], cb)]
+        out[it] = [inf['state_name'], bool(good)]
+    out['latest'] = list(pcc.latest({shm!r}))
+print(json.dumps(out))
+"""
+    env = dict(os.environ, PCC_FAULT="k1_fail:3")
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=600, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    res = json.loads(r.stdout.strip().splitlines()[-1])
+    states = [res[str(i)][0] for i in (10, 20, 30, 40)]
+    assert states.count("FAILED") == 1, res
+    for it in (10, 20, 30, 40):
+        if res[str(it)][0] != "FAILED":
+            assert res[str(it)] == ["LOCAL_COMMIT", True], res
+    assert res["latest"] == [40, 40]
+    rc, it, bad, outs = oracle.restore([shm], 3, [s.nbytes for s in config_tensors("c1")],
+                                       [s.code for s in config_tensors("c1")], 256, 4 << 20)
+    assert rc == 0 and it == 40
