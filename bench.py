@@ -1,18 +1,24 @@
 #!/usr/bin/env python
 """bench.py — snapshot GB/s of the PCcheck path on B200 (BASELINE.json metric).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--impl reference]
 
-A step is one whole checkpoint through pccheck.h — every row of SURVEY §8(a): the U-gate
-event, Listing 1 lines 3-11, K1 (gather-pack + CRC32C into the HBM ring), the finalize
-kernel (chunk CRCs + slice digest), copy-engine D2H straight into the registered DRAM
-file mapping (/dev/shm), header COMPLETE, the CAS commit and the pointer record, plus
-(N > 1) the NCCL allreduce(MIN) global commit.  K checkpoints are issued back to back
-with N = 2 in flight and the clock stops when the last one committed.
+A step is one whole checkpoint through pccheck.h — every row of SURVEY §8(a): the U-gate,
+Listing 1 lines 3-11, K1 (gather-pack + CRC32C into the HBM ring), the finalize kernels
+(chunk CRCs + slice digest), copy-engine D2H straight into the registered DRAM-file mapping
+(/dev/shm: the box has no NVMe), header COMPLETE, the CAS commit and the pointer record,
+plus (N > 1) the NCCL allreduce(MIN) global commit.  K checkpoints are issued back to back
+with N in flight and the clock stops when the last one committed.
+
+Default workload: BASELINE configs[2] — OPT-1.3B fp32 params + Adam (15.79 GB, 1552 tensors),
+64 MiB chunks, 4 in flight: the largest configuration that fits one GPU (configs[3]/[4] need
+2-8 GPUs; --config c4 / --gpus N runs them).
 
 value = state bytes of the whole job / time (box GB/s; per GPU = value / n_gpus).
 e2e   = the same with the state re-uploaded from pinned host memory every step.
-Rank 0 prints ONE JSON line.  --impl reference times the CPU oracle (oracle/) instead.
+--gpus N without torchrun: the bench starts N local rank processes itself (one per GPU) and
+fails loudly when fewer than N GPUs are visible.  Rank 0 prints ONE JSON line.
+--impl reference times the CPU oracle (oracle/) instead.
 """
 from __future__ import annotations
 
@@ -34,7 +40,8 @@ METRIC = "snapshot GB/s per GPU & box at 1/2/4/8 B200; % iter slowdown @ ckpt ev
 WORKLOADS = {
     "c1": "synthetic 64 MiB fp32 state in 97 mixed-size tensors, 4 MiB chunks, 2 in-flight checkpoints, DRAM-file target",
     "c2": "VGG-16 fp32 params + SGD momentum (1.107 GB), 16 MiB chunks, 2 in-flight checkpoints, DRAM-file target",
-    "c3": "OPT-1.3B fp32 params + Adam (15.79 GB), 64 MiB chunks, 4 in-flight checkpoints, DRAM-file target",
+    "c3": "OPT-1.3B fp32 params + Adam (15.79 GB, 1552 tensors), 64 MiB chunks, 4 in-flight checkpoints, "
+          "DRAM-file target (/dev/shm: the box has no NVMe SSD)",
     "c4": "BLOOM-7b1 bf16 params + fp32 master + Adam (98.97 GB), 64 MiB chunks, 1/world slice per rank",
     "bert": "BERT-large QA fp32 params + Adam (PAPER Table 3's 4 GB checkpoint), 64 MiB chunks, 2 in-flight "
             "checkpoints, DRAM-file target",
@@ -148,28 +155,28 @@ def bidir_peak_gbs(torch, nbytes=1 << 30):
     return nbytes / (best * 1e-3) / 1e9
 
 
-def cpu_baseline(specs, state, cb, budget_bytes=2 << 30, threads=1, hb=None):
+def cpu_baseline(specs, state, cb, budget_bytes=4 << 30, threads=1):
     """The oracle as it stands (plain C: byte-loop pack + byte-at-a-time CRC32C) on a bounded
-    sample: pack calls over the first chunks of the same image, up to `budget_bytes` (the whole
-    image for VGG-16), then the per-chunk CRCs.  threads > 1: that many host threads over
-    disjoint chunk ranges (K independent oracles; ctypes drops the GIL)."""
+    sample of the same image: its first chunks up to `budget_bytes` (the whole image when it is
+    smaller), then the per-chunk CRCs.  Each oracle is handed only the tensors overlapping its
+    chunk range (their bytes copied to the host by torch, untimed).  threads > 1: that many host
+    threads over disjoint chunk ranges, each an independent oracle (K independent
+    oracles; ctypes drops the GIL)."""
     import oracle
     from concurrent.futures import ThreadPoolExecutor
     from synth import host_bytes
-    hb = hb if hb is not None else [host_bytes(t) for t in state]
     nb = [s.nbytes for s in specs]
     off, end, c = oracle.layout(nb, 256, cb)
     k = max(1, min(c, budget_bytes // cb))
     parts = [(i * k // threads, (i + 1) * k // threads) for i in range(threads)]
     parts = [(a, b) for a, b in parts if b > a]
+    hi_all = k * cb
+    hb = {i: host_bytes(state[i]) for i in range(len(nb)) if nb[i] and int(off[i]) < hi_all}
 
     def run(ab):
-        if threads == 1:
-            img = oracle.pack(hb, 256, cb, first_chunk=ab[0], count=ab[1] - ab[0])
-        else:  # an independent oracle per range, handed only the tensors overlapping it
-            lo, hi = ab[0] * cb, ab[1] * cb
-            mine = {i: hb[i] for i in range(len(nb)) if int(off[i]) < hi and int(off[i]) + nb[i] > lo and nb[i]}
-            img = oracle.pack_chunks_sparse(nb, mine, 256, cb, ab[0], ab[1] - ab[0])
+        lo, hi = ab[0] * cb, ab[1] * cb
+        mine = {i: hb[i] for i in hb if int(off[i]) < hi and int(off[i]) + nb[i] > lo}
+        img = oracle.pack_chunks_sparse(nb, mine, 256, cb, ab[0], ab[1] - ab[0])
         oracle.chunk_crcs(img, cb)
 
     t0 = time.perf_counter()
@@ -178,7 +185,8 @@ def cpu_baseline(specs, state, cb, budget_bytes=2 << 30, threads=1, hb=None):
     dt = time.perf_counter() - t0
     return {"value": k * cb / dt / 1e9, "unit": "GB/s", "cores": len(parts), "kind": "oracle",
             "sample": f"pack + CRC32C of chunks 0..{k - 1} of {c} ({cb >> 20} MiB) of the same image "
-                      f"({k * cb / 1e9:.3f} GB, {dt:.1f} s, plain C, {len(parts)} thread(s) over disjoint chunk ranges)",
+                      f"({k * cb / 1e9:.3f} GB{' = the whole image' if k == c else ' prefix'}, {dt:.1f} s, plain C, "
+                      f"{len(parts)} thread(s) over disjoint chunk ranges)",
             "cpu": _cpu_model(), "nproc": os.cpu_count()}
 
 
@@ -203,6 +211,28 @@ def load_traffic(name):
         return None
 
 
+def default_inflight(cfg):
+    """N (Table 2: 2-4): 4 for OPT-1.3B (configs[2] says so), 2 elsewhere."""
+    return 4 if cfg == "c3" else 2
+
+
+def spawn_local_ranks(args):
+    """`python bench.py --gpus N` outside torchrun: start N rank processes on this node (one per
+    GPU, RANK / LOCAL_RANK / WORLD_SIZE / MASTER_* in their environment), wait for all, return
+    the worst exit code.  Rank 0 prints the JSON line."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    procs = []
+    for r in range(args.gpus):
+        env = dict(os.environ, RANK=str(r), LOCAL_RANK=str(r), WORLD_SIZE=str(args.gpus), LOCAL_WORLD_SIZE=str(args.gpus),
+                   MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        procs.append(subprocess.Popen([sys.executable, os.path.abspath(__file__)] + sys.argv[1:], env=env))
+    rcs = [p.wait() for p in procs]
+    return max(rcs, key=abs) if any(rcs) else 0
+
+
 def default_chunk_bytes(args):
     """chunk size b (R2): 4 MiB for the 64 MiB state; 16 MiB for VGG-16 (fig14 sweep: best of
     4/16/64/256 MiB — less zero padding in the last chunk); 64 MiB for the 10-100 GB states"""
@@ -212,31 +242,39 @@ def default_chunk_bytes(args):
 
 
 def run_reference(args, rank, world):
-    """--impl reference: the CPU oracle on the same workload, bounded sample per step."""
+    """--impl reference: the CPU oracle on the same workload, bounded sample per step (the next
+    ~128 MiB of chunks of the image per step); only the tensors a step's chunks overlap are
+    materialised (same seeded generator as the native arm, on the host)."""
     if rank != 0:
         return
-    import oracle  # noqa: F401  (reference arm: the one other place bench.py runs oracle/)
-    from synth import config_tensors
     import torch
+    import oracle as O  # the reference arm: the one other place bench.py runs oracle/
+    from synth import config_tensors, fill_tensor, torch_dtype
     specs = config_tensors(args.config)
     cb = default_chunk_bytes(args)
-    from synth import make_state
-    state = make_state(specs, "cpu", seed=0, it=0)
-    import oracle as O
-    hb = [t.reshape(-1).view(torch.uint8).numpy() if t.dim() else t.reshape(1).view(torch.uint8).numpy()
-          for t in state]
     nb = [s.nbytes for s in specs]
     off, end, c = O.layout(nb, 256, cb)
-    # a bounded sample per step: the next `per_step` chunks of the image (about 128 MiB), packed
-    # by an oracle handed only the tensors overlapping them (its pack walks every byte it is given)
     per_step = max(1, min(c, (128 << 20) // cb))
+    cache = {}
+
+    def host(i):  # tensor i as the native arm's make_state(seed=0, it=0) fills it, on the host
+        if i not in cache:
+            t = torch.empty(specs[i].shape, dtype=torch_dtype(specs[i].dtype))
+            fill_tensor(t, specs[i], 0, 0, i)
+            cache[i] = t.reshape(-1).view(torch.uint8).numpy() if t.dim() else t.reshape(1).view(torch.uint8).numpy()
+        return cache[i]
+
     times = []
     j = 0
     for step in range(args.warmup + args.steps):
         a = j % c
         k = min(per_step, c - a)
         lo, hi = a * cb, (a + k) * cb
-        mine = {i: hb[i] for i in range(len(nb)) if int(off[i]) < hi and int(off[i]) + nb[i] > lo and nb[i]}
+        idx = [i for i in range(len(nb)) if int(off[i]) < hi and int(off[i]) + nb[i] > lo and nb[i]]
+        for i in list(cache):
+            if i not in idx:
+                del cache[i]
+        mine = {i: host(i) for i in idx}
         t0 = time.perf_counter()
         img = O.pack_chunks_sparse(nb, mine, 256, cb, a, k)
         O.chunk_crcs(img, cb)
@@ -255,19 +293,67 @@ def run_reference(args, rank, world):
                        "chunk_bytes": cb},
             "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle",
                              "sample": f"per step: pack + CRC32C of the next {per_step} {cb >> 20} MiB chunks of the image "
-                                       f"(1 thread, plain C)"},
+                                       f"(1 thread, plain C; the tensors they overlap materialised untimed)"},
             "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def run_slowdowns(args, pcc, rank, world, coll, uid, peak_link, emu, torch, dist):
+    """The slowdown variants of the config's model (see the comment at the call site)."""
+    from tools import slowdown as S
+    kw = dict(iters=args.slowdown_iters, runs=args.slowdown_runs, every=10)
+    auto = dict(d2h_gbs="auto", link_gbs=peak_link)
+    plans = []
+    if args.config == "c2":
+        if world > 1:
+            ckw = dict(coll) if coll else {"nccl_unique_id": None}
+            for name, extra in (("slowdown", auto), ("slowdown_unpaced", {})):
+                def fn(extra=extra):
+                    if not coll:  # a fresh NCCL unique id per communicator, broadcast by torch
+                        obj = [pcc.nccl_unique_id() if rank == 0 else None]
+                        dist.broadcast_object_list(obj, src=0)
+                        ckw["nccl_unique_id"] = obj[0]
+                    return S.vgg16_slowdown(pcc, rank=rank, world=world, ck_kwargs=ckw, **kw, **extra)
+                plans.append((name, fn))
+        else:
+            plans = [("slowdown", lambda: S.vgg16_slowdown(pcc, graphs=True, **kw, **auto)),
+                     ("slowdown_eager", lambda: S.vgg16_slowdown(pcc, **kw, **auto)),
+                     ("slowdown_unpaced", lambda: S.vgg16_slowdown(pcc, **kw))]
+    elif args.config == "c3" and world == 1:
+        plans = [("slowdown", lambda: S.hf_slowdown(pcc, "opt13", graphs=True, n_inflight=args.inflight, **kw, **auto)),
+                 ("slowdown_eager", lambda: S.hf_slowdown(pcc, "opt13", n_inflight=args.inflight, **kw, **auto)),
+                 ("slowdown_unpaced", lambda: S.hf_slowdown(pcc, "opt13", n_inflight=args.inflight, **kw))]
+    elif args.config == "bert" and world == 1:
+        plans = [("slowdown", lambda: S.hf_slowdown(pcc, "bert", **kw, **auto)),
+                 ("slowdown_unpaced", lambda: S.hf_slowdown(pcc, "bert", **kw))]
+    elif args.config == "c4" and world == 1:
+        plans = [("slowdown", lambda: S.bloom_slowdown(pcc, world=emu or 8, **kw, **auto)),
+                 ("slowdown_unpaced", lambda: S.bloom_slowdown(pcc, world=emu or 8, **kw))]
+    out = {}
+    for name, fn in plans:
+        err = 0
+        try:
+            r = fn()
+        except Exception as ex:  # noqa: BLE001
+            r, err = {"error": repr(ex)[:300]}, 1
+        torch.cuda.empty_cache()
+        if world > 1:  # the max over ranks
+            t = torch.tensor([r.get("slowdown_pct") or 0.0, float(err)], device="cpu" if args.share_gpu else "cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            r["slowdown_pct_rank"] = r.get("slowdown_pct")
+            r["slowdown_pct"] = float(t[0]) if not float(t[1]) else None
+        out[name] = r
+    return out
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="c2")
+    ap.add_argument("--config", default="c3")
     ap.add_argument("--impl", default="native", choices=["native", "reference"])
-    ap.add_argument("--inflight", type=int, default=2)
+    ap.add_argument("--inflight", type=int, default=0, help="N checkpoints in flight (0 = per-config default)")
     ap.add_argument("--chunk-mib", type=int, default=0, help="chunk size b in MiB (0 = per-config default)")
     ap.add_argument("--ring-slices", type=int, default=2, help="HBM ring = this many slices")
     ap.add_argument("--d2h-gbs", type=float, default=0.0, help="pace the D2H copies (GB/s; 0 = full link)")
@@ -276,22 +362,32 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--mode", default="mapfile", choices=["mapfile", "zerocopy", "nullsink", "pwrite"])
     ap.add_argument("--share-gpu", action="store_true", help=argparse.SUPPRESS)  # test hook (see main)
-    ap.add_argument("--collectives", default="torch", choices=["torch", "nccl"],
-                    help="N>1: commit collectives via torch's NCCL process group (callbacks) or the library's own NCCL comm")
+    ap.add_argument("--collectives", default="nccl", choices=["torch", "nccl"],
+                    help="N>1: the library's own NCCL communicator (default) or torch.distributed callbacks")
+    ap.add_argument("--slowdown-iters", type=int, default=200, help="measured iterations per run (SURVEY §8(d): 200)")
+    ap.add_argument("--slowdown-runs", type=int, default=3, help="runs (PAPER L308: 3)")
     ap.add_argument("--emulate-world", type=int, default=0,
                     help="1 GPU plays rank 0 of this world size alone (PCC_NOCOMM): per-GPU share of a DP job")
     args = ap.parse_args()
+    args.inflight = args.inflight or default_inflight(args.config)
+    if args.impl == "reference":
+        run_reference(args, env_int("RANK", 0), env_int("WORLD_SIZE", 1))
+        return
+    if "RANK" not in os.environ and args.gpus > 1:  # not under torchrun: start the ranks ourselves
+        sys.exit(spawn_local_ranks(args))
     rank, world = env_int("RANK", 0), env_int("WORLD_SIZE", 1)
     local = env_int("LOCAL_RANK", 0)
-    if args.impl == "reference":
-        run_reference(args, rank, world)
-        return
+    if world != args.gpus:
+        sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}: refusing to report a "
+                 f"{world}-rank run as {args.gpus} GPUs")
     args.warmup = max(3, args.warmup)
 
     import torch
     import torch.distributed as dist
     if args.share_gpu:  # test hook: every rank on cuda:0, gloo transport (NCCL refuses duplicate GPUs)
         local = 0
+    elif torch.cuda.device_count() < world:
+        sys.exit(f"bench.py: {world} ranks need {world} GPUs, {torch.cuda.device_count()} visible")
     torch.cuda.set_device(local)
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
@@ -312,20 +408,10 @@ def main():
         obj = [pcc.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
-    elif world > 1:  # NCCL through torch's process group, handed to the library as callbacks
-        cdev = "cpu" if args.share_gpu else "cuda"
-
-        def _allreduce(vals, is_max):
-            t = torch.tensor(vals, dtype=torch.int64, device=cdev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX if is_max else dist.ReduceOp.MIN)
-            return t.tolist()
-
-        def _allgather(b):
-            t = torch.frombuffer(bytearray(b), dtype=torch.uint8).to(cdev)
-            parts = [torch.empty_like(t) for _ in range(world)]
-            dist.all_gather(parts, t)
-            return b"".join(x.cpu().numpy().tobytes() for x in parts)
-        coll = dict(allreduce=_allreduce, allgather=_allgather)
+    elif world > 1:  # torch.distributed as the library's transport (gloo with --share-gpu)
+        if not args.share_gpu:
+            sys.exit("bench.py: --collectives torch needs --share-gpu (gloo); use the native NCCL default")
+        coll = pcc.torch_collectives(dist)
     from paper_conf_asplos_strati0k25_b200 import k_layout
     n_est = k_layout([(1 << 20, s.nbytes, s.code) for s in specs], 256, cb)[2]
     slice_est = -(-n_est // world) * cb
@@ -424,7 +510,7 @@ def main():
     e3 = torch.cuda.Event(enable_timing=True)
     e2.record(stream)
     hs2 = []
-    e2e_steps = args.steps if state_bytes < (8 << 30) else min(args.steps, 3)  # bounded for 10-100 GB states
+    e2e_steps = args.steps  # the same step count as `value`
     for _ in range(e2e_steps):
         for i, h_ in host_state.items():
             state[i].copy_(h_, non_blocking=True)
@@ -468,64 +554,27 @@ def main():
     # the oracle as it stands on the host cores, on the same image (before the slowdown runs free
     # the state)
     cpu = cpu_all = None
-    if rank == 0 and not args.no_cpu_baseline and args.config in ("c1", "c2", "c3"):
-        from synth import host_bytes
-        hb = [host_bytes(t) for t in state]
-        cpu = cpu_baseline(specs, state, cb, hb=hb)
-        cpu_all = cpu_baseline(specs, state, cb, hb=hb, threads=len(os.sched_getaffinity(0)))
-        del hb
+    if rank == 0 and not args.no_cpu_baseline and args.config in ("c1", "c2", "c3", "bert"):
+        cpu = cpu_baseline(specs, state, cb)
+        cpu_all = cpu_baseline(specs, state, cb, threads=len(os.sched_getaffinity(0)))
 
-    # training slowdown, checkpoint every 10 iterations (BASELINE metric, second half):
-    #   slowdown           eager training, D2H paced by the tuner (tuner.choose_pace) — the
-    #                      library configured for training
-    #   slowdown_unpaced   eager training, the configuration `value` was measured in
-    #   slowdown_graphs    training step as CUDA graphs (VGG-16: tuned pace; OPT-1.3B: unpaced, host <= 2 replays ahead)
-    #   world > 1 (C2): VGG-16 under DDP on every rank, each checkpointing its 1/world slice with
-    #                      the collective commit; the slowdown reported is the max over ranks
-    slowdown = slowdown_unpaced = slowdown_graphs = None
-    if world > 1 and not args.no_slowdown and args.config == "c2":
-        from tools.slowdown import vgg16_slowdown
-        ckw = dict(coll) if coll else {"nccl_unique_id": uid}
-        res = {}
-        for name, kw in (("slowdown", dict(d2h_gbs="auto", link_gbs=peak_link)), ("slowdown_unpaced", {})):
-            try:
-                r = vgg16_slowdown(pcc, iters=60, every=10, rank=rank, world=world, ck_kwargs=ckw, **kw)
-                err = 0
-            except Exception as ex:  # noqa: BLE001
-                r, err = {"error": repr(ex)[:300]}, 1
-            t = torch.tensor([r.get("slowdown_pct", 0.0), float(err)], device="cpu" if args.share_gpu else "cuda")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            r["slowdown_pct_rank"] = r.get("slowdown_pct")
-            r["slowdown_pct"] = float(t[0]) if not float(t[1]) else None  # max over ranks
-            res[name] = r
-        slowdown, slowdown_unpaced = res["slowdown"], res["slowdown_unpaced"]
-    if rank == 0 and world == 1 and not args.no_slowdown and args.config in ("c2", "c3", "c4", "bert"):
-        try:
-            if args.config in ("c3", "bert"):  # the model's own training loop (tools/slowdown.hf_slowdown)
-                del state, host_state
-                torch.cuda.empty_cache()
-                from tools.slowdown import hf_slowdown
-                m = {"c3": "opt13", "bert": "bert"}[args.config]
-                slowdown = hf_slowdown(pcc, m, d2h_gbs="auto", link_gbs=peak_link)
-                slowdown_unpaced = hf_slowdown(pcc, m)
-                if m == "opt13":  # the step as one CUDA graph: immune to the eager launch penalty
-                    from tools.opt_graph_slowdown import opt13_graph_slowdown
-                    torch.cuda.empty_cache()
-                    slowdown_graphs = opt13_graph_slowdown()
-            elif args.config == "c2":
-                from tools.slowdown import vgg16_slowdown
-                slowdown = vgg16_slowdown(pcc, iters=60, every=10, d2h_gbs="auto", link_gbs=peak_link)
-                slowdown_unpaced = vgg16_slowdown(pcc, iters=60, every=10)
-                slowdown_graphs = vgg16_slowdown(pcc, iters=60, every=10, d2h_gbs="auto", link_gbs=peak_link,
-                                                 graphs=True)
-            else:
-                del state, host_state
-                torch.cuda.empty_cache()
-                from tools.slowdown import bloom_slowdown
-                slowdown = bloom_slowdown(pcc, world=emu or 8, iters=40, every=10, d2h_gbs="auto", link_gbs=peak_link)
-                slowdown_unpaced = bloom_slowdown(pcc, world=emu or 8, iters=40, every=10)
-        except Exception as ex:  # noqa: BLE001
-            slowdown = {"error": repr(ex)[:300]}
+    # training slowdown, checkpoint every 10 iterations (BASELINE metric, second half), on the
+    # config's own model with SURVEY §8(d)'s protocol (tools/slowdown.run_protocol: 20 warm-up +
+    # --slowdown-iters x --slowdown-runs, p50/p99, final drain):
+    #   slowdown           the library as configured for training: the tuner's D2H pace
+    #                      (tuner.choose_pace) — OPT-1.3B / VGG-16: step as 2 CUDA graphs
+    #   slowdown_eager     eager PyTorch, tuned pace
+    #   slowdown_unpaced   eager PyTorch, unpaced (the transfer configuration `value` is measured in)
+    #   world > 1: DDP on every rank, each checkpointing its 1/world slice with the collective
+    #   commit; the reported slowdown is the max over ranks
+    if "state" in locals():
+        del state
+    if "host_state" in locals():
+        del host_state
+    torch.cuda.empty_cache()
+    slowdowns = {}
+    if not args.no_slowdown:
+        slowdowns = run_slowdowns(args, pcc, rank, world, coll, uid, peak_link, emu, torch, dist)
 
     if rank == 0:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -575,9 +624,7 @@ def main():
                     "frac_of_bidir": e2e_value / world / peak_bidir},  # per GPU
             "gpu_launches": launches,
             "clocks": clk,
-            "slowdown": slowdown,
-            "slowdown_unpaced": slowdown_unpaced,
-            "slowdown_graphs": slowdown_graphs,
+            **slowdowns,
             "wall_s_timed": wall,
         }
         print(json.dumps(line), flush=True)

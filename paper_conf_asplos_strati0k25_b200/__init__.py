@@ -171,8 +171,11 @@ class PCCheck:
     def __init__(self, path=None, chunk_bytes=64 << 20, max_inflight=2, staging_bytes=0, ring_bytes=0,
                  writer_threads=4, flags=MAPFILE, device=0, rank=0, world=1, nccl_unique_id=None, align=256,
                  pack_ctas=0, allreduce=None, allgather=None, d2h_gbs=0.0, d2h_quantum=0):
-        """allreduce(values: list[int], is_max) -> list[int] and allgather(send: bytes) -> bytes
-        (rank-ordered concatenation) replace NCCL when given (e.g. torch.distributed gloo).
+        """allreduce(values: list[int], is_max) -> list[int] and allgather(send, recv) replace the
+        library's NCCL communicator when given (e.g. torch.distributed over gloo; see
+        ``torch_collectives``).  allgather gets zero-copy numpy uint8 views of the library's pinned
+        buffers — send (n bytes) and recv (world * n bytes, rank-ordered) — and fills recv in place,
+        so no chunk bytes are copied through Python objects.
         d2h_gbs / d2h_quantum: pace the copy-engine D2H (GB/s, bytes per copy; 0 = unpaced)."""
         self._uid = None
         self._cbs = None
@@ -190,10 +193,15 @@ class PCCheck:
             cbs.append(ALLREDUCE_FN(_ar))
             ar = C.cast(cbs[-1], C.c_void_p)
         if allgather is not None:
+            import numpy as np
+
+            def _view(ptr, n):
+                return np.ctypeslib.as_array(C.cast(ptr, C.POINTER(C.c_uint8)), shape=(n,)) if n else \
+                    np.empty(0, dtype=np.uint8)
+
             def _ag(ctx, send, recv, nbytes):
                 try:
-                    data = allgather(C.string_at(send, nbytes))
-                    C.memmove(recv, data, len(data))
+                    allgather(_view(send, nbytes), _view(recv, nbytes * world))
                     return 0
                 except Exception:  # noqa: BLE001
                     return 1
@@ -286,6 +294,26 @@ class PCCheck:
             self.close()
         except Exception:
             pass
+
+
+def torch_collectives(dist, group=None):
+    """allreduce / allgather callbacks for ``PCCheck`` over an initialised torch.distributed
+    CPU process group (gloo) — the transport for tests that run several ranks on one GPU, where
+    NCCL cannot.  Marshalling only: allgather hands zero-copy tensors over the library's pinned
+    buffers to ``dist.all_gather``."""
+    import torch
+    world = dist.get_world_size(group)
+
+    def allreduce(vals, is_max):
+        t = torch.tensor(vals, dtype=torch.int64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX if is_max else dist.ReduceOp.MIN, group=group)
+        return t.tolist()
+
+    def allgather(send, recv):
+        st = torch.from_numpy(send)
+        dist.all_gather(list(torch.from_numpy(recv).view(world, -1).unbind(0)), st, group=group)
+
+    return dict(allreduce=allreduce, allgather=allgather)
 
 
 _STATE_KEYS = ("momentum_buffer", "exp_avg", "exp_avg_sq", "step")

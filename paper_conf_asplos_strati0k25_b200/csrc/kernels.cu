@@ -229,6 +229,14 @@ __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_gr
 __device__ __forceinline__ void prefetch_l2(uint64_t addr) {
     asm volatile("prefetch.global.L2 [%0];" ::"l"(addr));
 }
+__device__ __forceinline__ void prefetch_l2_bulk(uint64_t addr, uint32_t bytes) {  // addr, bytes: 16-B multiples
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(addr), "r"(bytes) : "memory");
+}
+// A/B hook: the round-ahead L2 prefetch as ONE bulk prefetch per warp when the round is one
+// contiguous source range (PCC_PF2_BULK=1) instead of 32 per-lane prefetches
+#ifndef PCC_PF2_BULK
+#define PCC_PF2_BULK 0
+#endif
 
 struct Span {  // one lane's 32 bytes of a round
     uint4 a, b;
@@ -304,7 +312,20 @@ __device__ __forceinline__ void tile_fast(const char *ntab, const char *nf, char
         if (kPf2Of<kPack> && r + kAhead + 1 < kRounds) {
             if (kPack) {
                 uint64_t a = 0;
-                if (rc.at(pos(r + kAhead + 1), a)) prefetch_l2(a);
+                const uint32_t k = rc.at(pos(r + kAhead + 1), a);
+#if PCC_PF2_BULK
+                // one TMA bulk prefetch per warp when the round's 1 KiB is one contiguous source
+                // range (the common case: inside one big tensor), else one prefetch per lane
+                const uint64_t a0 = __shfl_sync(0xFFFFFFFFu, a, 0);
+                const bool contig = __all_sync(0xFFFFFFFFu, k == 16 && a == a0 + lane * kLaneSpan && (a0 & 15) == 0);
+                if (contig) {
+                    if (lane == 0) prefetch_l2_bulk(a0, kRound);
+                } else if (k) {
+                    prefetch_l2(a);
+                }
+#else
+                if (k) prefetch_l2(a);
+#endif
             } else {
                 prefetch_l2(reinterpret_cast<uint64_t>(chunk + pos(r + kAhead + 1)));
             }
@@ -400,10 +421,6 @@ __device__ __forceinline__ uint2 item_rows(const SnapParams &P, uint32_t item, u
     if (item >= n_items) return make_uint2(0, 0);
     const uint32_t jl = item / P.tpc, t = item - jl * P.tpc;
     return __ldg(P.tile_rows + (uint64_t)(P.first + jl) * P.tpc + t);
-}
-
-__device__ __forceinline__ void prefetch_l2_bulk(uint64_t addr, uint32_t bytes) {  // addr, bytes: 16-B multiples
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(addr), "r"(bytes) : "memory");
 }
 
 // Warm L2 with the bytes of the warp's NEXT work item while it works on this one (a TMA bulk

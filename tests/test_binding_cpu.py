@@ -38,3 +38,43 @@ def test_state_tensors_rejects_host_state_of_device_params():
     p = torch.nn.Parameter(torch.zeros(2, device="meta"))
     with pytest.raises(ValueError):
         pcc.state_tensors(FakeOpt(p))
+
+
+def _coll_worker(rank, world, port, q):
+    import os
+    import numpy as np
+    import torch.distributed as dist
+    import paper_conf_asplos_strati0k25_b200 as pcc
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        coll = pcc.torch_collectives(dist)
+        assert coll["allreduce"]([rank + 5, -rank], True) == [world + 4, 0]
+        assert coll["allreduce"]([rank + 5, -rank], False) == [5, -(world - 1)]
+        n = 1 << 20  # one MiB per rank, written in place into the receive view
+        send = np.full(n, 17 + rank, dtype=np.uint8)
+        recv = np.zeros(world * n, dtype=np.uint8)
+        coll["allgather"](send, recv)
+        ok = all((recv[r * n:(r + 1) * n] == 17 + r).all() for r in range(world))
+        coll["allgather"](np.empty(0, np.uint8), np.empty(0, np.uint8))  # zero bytes per rank
+        q.put((rank, bool(ok)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_torch_collectives_gloo_world2():
+    """The zero-copy gloo adapter the DP tests and the binding use for caller collectives:
+    allreduce MIN/MAX and an in-place rank-ordered allgather into the receive view."""
+    import os
+    import torch.multiprocessing as mp
+    port = 31000 + os.getpid() % 2000
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_coll_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    for p in ps:
+        p.join(120)
+        assert p.exitcode == 0
+    assert sorted(q.get(timeout=10) for _ in range(2)) == [(0, True), (1, True)]

@@ -36,19 +36,8 @@ torch.cuda.set_device(0)
 specs = config_tensors("c1")
 ts = make_state(specs, "cuda", seed=51, it=0)
 
-def allreduce(vals, is_max):
-    t = torch.tensor(vals, dtype=torch.int64)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX if is_max else dist.ReduceOp.MIN)
-    return t.tolist()
-
-def allgather(b):
-    t = torch.frombuffer(bytearray(b), dtype=torch.uint8)
-    parts = [torch.empty_like(t) for _ in range(world)]
-    dist.all_gather(parts, t)
-    return b"".join(p.numpy().tobytes() for p in parts)
-
 ck = pcc.PCCheck(os.path.join(d, f"r{rank}.pcc"), chunk_bytes=4 << 20, max_inflight=2,
-                 flags=pcc.MAPFILE | pcc.FSYNC, rank=rank, world=world, allreduce=allreduce, allgather=allgather)
+                 flags=pcc.MAPFILE | pcc.FSYNC, rank=rank, world=world, **pcc.torch_collectives(dist))
 ck.register(ts)
 if mode == "crash":
     for it in (10, 20):

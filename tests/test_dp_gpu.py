@@ -28,21 +28,10 @@ def _rank_main(rank, world, tmpdir, port, q):
         specs = config_tensors("c1")
         ts = make_state(specs, "cuda", seed=31, it=0)  # replicated DP state: same seed on every rank
 
-        def allreduce(vals, is_max):
-            t = torch.tensor(vals, dtype=torch.int64)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX if is_max else dist.ReduceOp.MIN)
-            return t.tolist()
-
-        def allgather(b):
-            t = torch.frombuffer(bytearray(b), dtype=torch.uint8)
-            parts = [torch.empty_like(t) for _ in range(world)]
-            dist.all_gather(parts, t)
-            return b"".join(p.numpy().tobytes() for p in parts)
-
         path = os.path.join(tmpdir, f"r{rank}.pcc")
         saved = {}
         with pcc.PCCheck(path, chunk_bytes=CB, max_inflight=2, flags=pcc.MAPFILE, rank=rank, world=world,
-                         allreduce=allreduce, allgather=allgather) as ck:
+                         **pcc.torch_collectives(dist)) as ck:
             ck.register(ts)
             geo = ck.geometry()
             out["slice"] = (geo["first"], geo["count"], geo["n_chunks"])

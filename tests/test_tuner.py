@@ -68,3 +68,44 @@ def test_tune_live_c1():
     assert set(out["Tw_by_N"]) == {1, 2, 3, 4}
     assert all(v > 0 for v in out["Tw_by_N"].values())
     assert 1 <= out["N"] <= 4 and out["f"] >= 1
+
+
+def test_choose_chunk_tg_and_padding():
+    """b from T_G (L176): a faster link rate wins, but zero padding (R3) counts against big b."""
+    from paper_conf_asplos_strati0k25_b200.tuner import choose_chunk
+    MiB = 1 << 20
+    tg = {4 * MiB: 50.0, 16 * MiB: 55.0, 64 * MiB: 56.0, 256 * MiB: 56.0}
+    # VGG-16's 1.107 GB state: 64 MiB pads the last chunk by 3.0%, 16 MiB by 0.04%
+    out = choose_chunk(tg, 1_106_860_352)
+    assert out["chunk_bytes"] == 16 * MiB
+    assert out["eff_by_b"][64 * MiB] == pytest.approx(56.0 * 1_106_860_352 / (17 * 64 * MiB))
+    # a state of exactly 16 x 64 MiB: no padding anywhere, 64 MiB's faster link wins over 16 MiB
+    out = choose_chunk(tg, 16 * 64 * MiB, tol=0.995)
+    assert out["chunk_bytes"] == 64 * MiB
+    # tolerance: the smallest b within 3% of the best
+    assert choose_chunk({1: 97.0, 2: 100.0}, 2)["chunk_bytes"] == 1
+    with pytest.raises(ValueError):
+        choose_chunk({}, 1)
+
+
+def test_choose_ring_variants():
+    from paper_conf_asplos_strati0k25_b200.tuner import choose_ring
+    GB, MiB = 10 ** 9, 1 << 20
+    s = 12_348_030_976  # BLOOM-7b1 rank slice at W = 8 (185 x 64 MiB)
+    # plenty of HBM: the whole slice (x N in flight, capped at N slices)
+    r = choose_ring(s, 64 * MiB, 40 * GB, 2, 55.0)
+    assert r["variant"] == "B" and r["ring_chunks"] == 2 * 184 and r["stall_s"] < 0.01
+    # a 4 GB budget: windowed ring, stall = pack + the part beyond the ring over the link
+    r = choose_ring(s, 64 * MiB, 4 * GB, 2, 55.0)
+    assert r["variant"] == "B" and r["ring_chunks"] == 59
+    assert r["stall_s"] == pytest.approx(2 * s / 5e12 + (s - 59 * 64 * MiB) / 55e9)
+    assert r["stall_s"] < r["stall_s_A"]
+    # no HBM to spare: Variant A (K1 stores into host memory, the U-gate spans the transfer)
+    r = choose_ring(s, 64 * MiB, 32 * MiB, 2, 55.0)
+    assert r["variant"] == "A" and r["ring_bytes"] == 0 and r["stall_s"] == pytest.approx(s / (0.92 * 55e9))
+
+
+def test_pace_delivery():
+    from paper_conf_asplos_strati0k25_b200.tuner import pace_delivery
+    assert pace_delivery(27.0, 28.5) == pytest.approx(0.947, rel=1e-3)
+    assert pace_delivery(0.0, 28.5) is None and pace_delivery(27.0, 0.0) is None
