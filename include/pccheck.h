@@ -176,19 +176,20 @@ PCC_API int pcc_register(pcc_ctx *ctx, const pcc_tensor *t, uint32_t n);
 /* Starts checkpoint `iter` of the registered state as it is on `train_stream` now.
  * Listing 1 lines 3-11 (sample the pointer, take the counter, dequeue a free slot — this
  * BLOCKS while N checkpoints hold all N+1 slots, the paper's stall, L139 Fig 6), records an
- * event on train_stream and hands the checkpoint to the library's threads: the packer launches
- * K1 on the pack stream after that event (in windows, as HBM ring space frees), the
- * orchestrator streams the chunks to host memory.  It never waits for ring space or for an
- * earlier checkpoint's transfer.  iter must strictly increase (-PCC_EORDER).  *out receives
- * the handle.  World > 1: COLLECTIVE when a rank has no free slot (backpressure rounds). */
+ * event on train_stream, and enqueues K1 on the library's pack stream behind that event when
+ * the HBM ring has room for the slice; otherwise hands the checkpoint to the library's packer
+ * thread, which launches K1 in windows as ring space frees.  It never waits for ring space or
+ * for an earlier checkpoint's transfer.  iter must strictly increase (-PCC_EORDER).  *out
+ * receives the handle.  World > 1: COLLECTIVE when a rank has no free slot (backpressure). */
 PCC_API int pcc_checkpoint(pcc_ctx *ctx, uint64_t iter, void *train_stream, pcc_handle *out);
 
-/* U-gate (L139): makes train_stream wait until the newest checkpoint's K1 finished reading
- * the registered tensors.  Call before the optimizer step that overwrites them.  The wait is
- * on the GPU (cuStreamWaitValue32 on a word the pack stream writes after the checkpoint's
- * last K1 window): the call returns at once even if K1 has not been launched yet.  Without
- * stream memory operations (or with PCC_NO_STREAM_MEMOPS set) the host waits until the K1
- * windows are enqueued, then the stream waits for their event.  No-op before any checkpoint. */
+/* U-gate (L139): makes train_stream wait (cudaStreamWaitEvent) until the newest checkpoint's
+ * K1 finished reading the registered tensors.  Call before the optimizer step that overwrites
+ * them.  Returns at once when that checkpoint's K1 windows are enqueued; when the packer thread
+ * still holds some (ring space), it first waits on the host until they are — the training
+ * stream is only ever made to wait for work already on the GPU (a stream-side wait for work
+ * another thread enqueues later deadlocks under lazy module loading and pageable copies,
+ * profiles/r02_gate_probe_*.txt).  No-op before any checkpoint. */
 PCC_API int pcc_guard(pcc_ctx *ctx, void *train_stream);
 
 PCC_API int pcc_poll(pcc_ctx *ctx, pcc_handle h, int *state);

@@ -67,5 +67,8 @@ cudaError_t launch_pack(const SnapParams &p, int grid, cudaStream_t s);
 cudaError_t launch_unpack(const SnapParams &p, int grid, cudaStream_t s);
 cudaError_t launch_finalize(const FinalizeParams &p, cudaStream_t s);  // kFinalizeLaunches kernels
 constexpr int kFinalizeLaunches = 2;
+// One no-work launch of each pipeline kernel (+ its launch attributes) so that lazy module
+// loading happens at open time, not inside a checkpoint.  Synchronous.
+cudaError_t warm_kernels(int device, const CrcTables *tables);
 
 }  // namespace pcc

@@ -14,7 +14,6 @@
 // Chunks of a checkpoint land contiguously in their slot (L127, L281: "contiguous on
 // storage"), N checkpoints may be in flight (L139, Fig 6), copy and persist overlap per
 // chunk (L141, Fig 7).
-#include <cuda.h>  // driver-API types for the stream memory operations (fetched via cudart, no -lcuda)
 #include <cuda_runtime.h>
 #include <fcntl.h>
 #include <sys/mman.h>
@@ -66,34 +65,6 @@ struct NvtxRange {
     NvtxRange &operator=(const NvtxRange &) = delete;
 };
 
-// Stream memory operations (cuStreamWaitValue32 / cuStreamWriteValue32), fetched from the
-// driver through cudart so the library needs no -lcuda.  The U-gate uses them: the training
-// stream waits ON THE GPU for a word the pack stream writes after a checkpoint's last K1 window,
-// so pcc_checkpoint / pcc_guard never block the calling thread on ring space.
-using WaitValue32Fn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
-using WriteValue32Fn = CUresult (*)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
-struct StreamMemOps {
-    WaitValue32Fn wait32 = nullptr;
-    WriteValue32Fn write32 = nullptr;
-    bool ok() const { return wait32 && write32; }
-};
-static const StreamMemOps &stream_mem_ops() {
-    static const StreamMemOps ops = [] {
-        StreamMemOps o;
-        if (std::getenv("PCC_NO_STREAM_MEMOPS")) return o;  // test hook: the host-blocking fallback
-        cudaDriverEntryPointQueryResult q1 = cudaDriverEntryPointSymbolNotFound, q2 = q1;
-        void *w = nullptr, *x = nullptr;
-        if (cudaGetDriverEntryPointByVersion("cuStreamWaitValue32", &w, 12000, cudaEnableDefault, &q1) == cudaSuccess &&
-            cudaGetDriverEntryPointByVersion("cuStreamWriteValue32", &x, 12000, cudaEnableDefault, &q2) == cudaSuccess &&
-            q1 == cudaDriverEntryPointSuccess && q2 == cudaDriverEntryPointSuccess) {
-            o.wait32 = reinterpret_cast<WaitValue32Fn>(w);
-            o.write32 = reinterpret_cast<WriteValue32Fn>(x);
-        }
-        return o;
-    }();
-    return ops;
-}
-
 // PCC_TRACE=1: one stderr line per pipeline event (debugging hangs on the GPU box)
 static bool trace_on() {
     static int on = -1;
@@ -115,7 +86,7 @@ struct Launch {
 
 struct Ckpt {
     Ticket t;
-    uint32_t seq = 0;  // 1, 2, ... in pcc_checkpoint order: the U-gate word value after its last K1
+    uint32_t seq = 0;  // 1, 2, ... in pcc_checkpoint order (U-gate bookkeeping)
     std::atomic<int> state{PCC_ST_QUEUED};
     std::atomic<int> err{0};
     std::atomic<bool> packed_recorded{false};  // ev_packed recorded by the packer thread
@@ -225,10 +196,13 @@ struct pcc_ctx {
     std::mutex ring_mu;
     std::condition_variable ring_cv;
 
-    // U-gate: device word written (stream-ordered) after each checkpoint's last K1 window
-    uint32_t *gate_dev = nullptr;
+    // U-gate bookkeeping.  The training stream may only ever wait for GPU work that is ALREADY
+    // enqueued (an event): a stream-side wait for work another host thread enqueues later
+    // deadlocks under PyTorch's lazy module loading and while any thread sits in a pageable
+    // memcpy, which holds a process-wide driver lock (profiles/r02_gate_probe_*.txt).
     uint32_t issued_seq = 0;                 // caller thread: seq of the newest pcc_checkpoint
-    std::atomic<uint32_t> packed_seq{0};     // packer: seq whose K1 windows + gate write are enqueued
+    std::atomic<uint32_t> packed_seq{0};     // seq whose K1 windows + ev_guard are enqueued
+    uint32_t handed_seq = 0;                 // caller thread: newest seq handed to the packer thread
     std::mutex pk_mu;
     std::condition_variable pk_cv;
 
@@ -480,7 +454,10 @@ void orchestrate_loop(pcc_ctx *c) {
         PCC_TRACE("orch: ckpt %llu iter %llu slot %u", (unsigned long long)ck->t.counter,
                   (unsigned long long)ck->t.iter, ck->t.slot);
         NvtxRange nv("pcc.d2h");
-        // (the FILLING header of R18 was written by the packer before its first K1 launch)
+        if (c->fd >= 0 && !c->zerocopy()) {
+            int rc = c->engine->filling(ck->t);  // R18: before any data byte of this slot changes
+            if (rc) fail_ckpt(c, ck, rc);
+        }
         size_t li = 0;
         uint32_t issued = 0;
         // D2H pacing (pcc_config d2h_mbps / d2h_quantum): copies of at most `quantum` bytes,
@@ -664,20 +641,20 @@ bool any_inflight(pcc_ctx *c) {
     return false;
 }
 
-// The packer thread: K1 for one checkpoint, after the caller's event on the training stream.
-// Runs checkpoints strictly in pcc_checkpoint order, so K1 windows, the U-gate word and the
-// finalize kernels are stream-ordered on the pack stream.  Waiting for HBM ring space
-// (Variant B with a ring smaller than the slices in flight) happens HERE, not in the caller:
-// the training thread only enqueues, and the U-gate holds the training
-// stream on the GPU instead (pcc_guard).
+// K1 for one checkpoint, after the caller's event on the training stream: run inline by
+// pcc_checkpoint when the ring already has room, else by the packer thread, strictly in
+// checkpoint order either way, so K1 windows, ev_guard and the finalize kernels of successive
+// checkpoints are stream-ordered on the pack stream.  Waiting for HBM ring space (Variant B
+// with a ring smaller than the slices in flight) happens in the packer thread, never in the
+// caller's pcc_checkpoint.
 void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
     NvtxRange nv("pcc.pack");
     const uint32_t s = ck->t.slot;
     cudaStreamWaitEvent(c->pack_stream, ck->ev_train, 0);
-    if (c->fd >= 0) {
-        // R18: the reused slot's header becomes FILLING before any data byte of the slot changes
-        // — before K1 is even launched, which matters in ZEROCOPY mode where K1 stores straight
-        // into the slot's file pages
+    if (c->fd >= 0 && c->zerocopy()) {
+        // R18: the reused slot's header becomes FILLING before any data byte of the slot changes.
+        // In ZEROCOPY mode K1 itself stores into the slot's file pages, so this happens before K1
+        // is launched; otherwise the orchestrator writes it before its first D2H.
         int rc = c->engine->filling(ck->t);
         if (rc) fail_ckpt(c, ck, rc);
     }
@@ -756,17 +733,9 @@ void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
     }
     cudaEventRecord(ck->ev_packed, c->pack_stream);
     ck->packed_recorded = true;
-    // open the U-gate: stream-ordered after the last K1 window (written even when a launch
-    // failed, so a guarded training stream is never left waiting)
-    if (stream_mem_ops().ok())
-        stream_mem_ops().write32(reinterpret_cast<CUstream>(c->pack_stream), reinterpret_cast<CUdeviceptr>(c->gate_dev),
-                                 ck->seq, CU_STREAM_WRITE_VALUE_DEFAULT);
+    // the U-gate event: after the last K1 window (recorded even when a launch failed, so a
+    // guarded training stream is never left waiting)
     cudaEventRecord(c->ev_guard, c->pack_stream);
-    {
-        std::lock_guard<std::mutex> lk(c->pk_mu);
-        c->packed_seq.store(ck->seq);
-    }
-    c->pk_cv.notify_all();
     // chunk CRCs -> slice digest, then the table to pinned host memory for the header
     cudaMemsetAsync(c->scratch_dev[s], 0, 4 * sizeof(uint32_t), c->pack_stream);
     FinalizeParams F{};
@@ -795,6 +764,11 @@ void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
         }
     }
     ck->cv.notify_all();
+    {  // everything of this checkpoint is on the pack stream: pcc_guard may take ev_guard now
+        std::lock_guard<std::mutex> lk(c->pk_mu);
+        c->packed_seq.store(ck->seq);
+    }
+    c->pk_cv.notify_all();
 }
 
 void pack_loop(pcc_ctx *c) {
@@ -863,6 +837,10 @@ int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
     cudaError_t e = cudaSetDevice(c->device);
     if (e != cudaSuccess) return cuda_error(e, "cudaSetDevice");
     if ((e = device_tables(c->device, &c->tables, &c->consts)) != cudaSuccess) return cuda_error(e, "CRC tables");
+    // load every kernel the pipeline launches now, on the caller's thread: under lazy module
+    // loading (PyTorch's default) a first launch synchronises the context, which must not happen
+    // inside a checkpoint
+    if ((e = warm_kernels(c->device, c->tables)) != cudaSuccess) return cuda_error(e, "kernel warm-up");
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
     // PCC_PACK_PRIO=low|default (experiments): K1's stream priority relative to training
@@ -873,8 +851,6 @@ int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
     cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking);
     cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking);
     cudaEventCreateWithFlags(&c->ev_guard, cudaEventDisableTiming);
-    if ((e = cudaMalloc(&c->gate_dev, sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "U-gate word");
-    if ((e = cudaMemset(c->gate_dev, 0, sizeof(uint32_t))) != cudaSuccess) return cuda_error(e, "U-gate word");
     if (!nullsink) {
         int flags = O_RDWR | O_CREAT;
         if ((cfg->flags & PCC_ODIRECT) && !(cfg->flags & PCC_MAPFILE)) flags |= O_DIRECT;
@@ -1077,10 +1053,22 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
         c->ckpts[ck->t.counter] = ck;
     }
     c->guard_armed = true;
-    // K1 (packer thread) and the D2H (orchestrator) follow asynchronously; this call never
-    // waits for ring space or for the previous checkpoint's transfer
-    c->jobs.push(ck);
-    c->packs.push(ck);
+    c->jobs.push(ck);  // the orchestrator follows the K1 windows as they are published
+    // K1: enqueued right here when nothing is queued ahead of it and the HBM ring already has room
+    // for the whole slice (the usual case: the previous checkpoints drained within the interval);
+    // otherwise the packer thread launches the windows as ring space frees.  Either way this call
+    // never waits for ring space or for an earlier checkpoint's transfer.
+    bool inline_pack = !c->zerocopy() && (int32_t)(c->packed_seq.load() - c->handed_seq) >= 0;
+    if (inline_pack) {
+        std::lock_guard<std::mutex> lk(c->ring_mu);
+        inline_pack = c->ring_tail + c->ring_slots >= c->ring_head + c->n;
+    }
+    if (inline_pack) {
+        pack_one(c, ck);
+    } else {
+        c->handed_seq = ck->seq;
+        c->packs.push(ck);
+    }
     *out = ck->t.counter;
     return PCC_OK;
 }
@@ -1090,17 +1078,9 @@ int pcc_guard(pcc_ctx *c, void *train_stream) {
     if (!c->guard_armed) return PCC_OK;
     cudaStream_t ts = static_cast<cudaStream_t>(train_stream);
     const uint32_t want = c->issued_seq;
-    if (stream_mem_ops().ok()) {
-        // the training stream waits on the GPU until the pack stream wrote `want` — after the
-        // newest checkpoint's last K1 window, whenever the packer gets to launch it
-        CUresult r = stream_mem_ops().wait32(reinterpret_cast<CUstream>(ts), reinterpret_cast<CUdeviceptr>(c->gate_dev),
-                                             want, CU_STREAM_WAIT_VALUE_GEQ);
-        if (r != CUDA_SUCCESS) return set_error(PCC_ECUDA, "cuStreamWaitValue32 (U-gate)");
-        return PCC_OK;
-    }
-    // fallback without stream memory operations: the host waits until the packer enqueued the
-    // newest checkpoint's K1 windows, then the stream waits for their event (still exact)
-    {
+    // only when the packer thread still holds K1 windows of the newest checkpoint (ring space):
+    // wait here, on the host and outside any CUDA call, until they are enqueued
+    if ((int32_t)(c->packed_seq.load() - want) < 0) {
         std::unique_lock<std::mutex> lk(c->pk_mu);
         c->pk_cv.wait(lk, [&] { return (int32_t)(c->packed_seq.load() - want) >= 0; });
     }
@@ -1289,7 +1269,6 @@ int pcc_close(pcc_ctx *c) {
     free_registration(c);
     for (auto e : c->evpool) cudaEventDestroy(e);
     cudaEventDestroy(c->ev_guard);
-    if (c->gate_dev) cudaFree(c->gate_dev);
     cudaStreamDestroy(c->pack_stream);
     cudaStreamDestroy(c->copy_stream);
     cudaStreamDestroy(c->aux_stream);

@@ -130,5 +130,12 @@ int main() {
     run_bulk<4>(s, d, bytes, 32768, cps, nsm, st, bad, "4x32K");
     run_bulk<6>(s, d, bytes, 16384, cps, nsm, st, bad, "6x16K");
   }
+  // round 2: the staging K1 could afford next to its 193 KiB of CRC tables (~34 KiB per SM,
+  // one CTA per SM): is a TMA ring that small still at the copy peak?
+  run_bulk<4>(s, d, bytes, 8192, 1, nsm, st, bad, "4x8K_1cta_32KiB");
+  run_bulk<2>(s, d, bytes, 16384, 1, nsm, st, bad, "2x16K_1cta_32KiB");
+  run_bulk<8>(s, d, bytes, 4096, 1, nsm, st, bad, "8x4K_1cta_32KiB");
+  run_bulk<8>(s, d, bytes, 8192, 1, nsm, st, bad, "8x8K_1cta_64KiB");
+  run_bulk<8>(s, d, bytes, 16384, 1, nsm, st, bad, "8x16K_1cta_128KiB");
   return 0;
 }
