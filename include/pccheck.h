@@ -78,6 +78,13 @@ enum {
                                shard"): every rank registers its OWN tensors and checkpoints all
                                of them — no 1/world slicing, no restore fan-out; the global commit
                                and the restore agreement still run across ranks. */
+    PCC_D2H_UPFRONT = 1u << 7, /* the copy-engine D2H of each K1 window is enqueued by the thread
+                               that launches the window, at once (no pacing, no queue drains), so the
+                               transfer needs no later CUDA call from the library's threads.  For
+                               training loops run as CUDA graphs: a host thread blocked in
+                               cudaGraphLaunch (GPU queue full) stalls every other thread's CUDA calls
+                               for up to one replay.  Eager loops that read values to
+                               the host every step want the default (drained, optionally paced). */
 };
 
 /* ---- per-checkpoint states (pcc_poll) — SURVEY §8(b) state machine ------------------- */

@@ -24,7 +24,7 @@ _lib = C.CDLL(LIB_PATH)
 ABI_VERSION = 2
 NONE = LATEST = (1 << 64) - 1
 OK, EINVAL, ENOMEM, EBUSY, EAGAIN, EIO, ECUDA, ENCCL, EORDER, ECORRUPT, ELAYOUT, ENOENT, ETIMEDOUT, ESTATE = range(14)
-ODIRECT, FSYNC, ZEROCOPY, NULLSINK, MAPFILE, NOCOMM, SHARDED = 1, 2, 4, 8, 16, 32, 64
+ODIRECT, FSYNC, ZEROCOPY, NULLSINK, MAPFILE, NOCOMM, SHARDED, D2H_UPFRONT = 1, 2, 4, 8, 16, 32, 64, 128
 FALLBACK = 1
 (ST_QUEUED, ST_PACKING, ST_PACKED, ST_PERSISTED, ST_LOCAL_COMMIT, ST_GLOBAL_COMMIT, ST_OBSOLETE,
  ST_FAILED) = range(8)

@@ -71,12 +71,17 @@ static bool trace_on() {
     if (on < 0) on = std::getenv("PCC_TRACE") ? 1 : 0;
     return on;
 }
-#define PCC_TRACE(...)                        \
-    do {                                      \
-        if (trace_on()) {                     \
-            std::fprintf(stderr, "[pcc] " __VA_ARGS__); \
-            std::fputc('\n', stderr);         \
-        }                                     \
+static double trace_ms() {
+    static const auto t0 = std::chrono::steady_clock::now();
+    return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
+#define PCC_TRACE(...)                                             \
+    do {                                                           \
+        if (trace_on()) {                                          \
+            std::fprintf(stderr, "[pcc %10.3f] ", trace_ms());     \
+            std::fprintf(stderr, __VA_ARGS__);                     \
+            std::fputc('\n', stderr);                              \
+        }                                                          \
     } while (0)
 
 struct Launch {
@@ -244,6 +249,7 @@ struct pcc_ctx {
     bool mapfile() const { return cfg.flags & PCC_MAPFILE; }
     bool nullsink() const { return cfg.flags & PCC_NULLSINK; }
     bool zerocopy() const { return cfg.flags & PCC_ZEROCOPY; }
+    bool upfront() const { return (cfg.flags & PCC_D2H_UPFRONT) && !zerocopy(); }
     uint64_t cb() const { return cfg.chunk_bytes; }
     uint64_t slot_data_off(uint32_t s) const { return slot_offset(s, n, cb()) + header_bytes(n); }
 };
@@ -651,10 +657,11 @@ void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
     NvtxRange nv("pcc.pack");
     const uint32_t s = ck->t.slot;
     cudaStreamWaitEvent(c->pack_stream, ck->ev_train, 0);
-    if (c->fd >= 0 && c->zerocopy()) {
+    if (c->fd >= 0 && (c->zerocopy() || c->upfront())) {
         // R18: the reused slot's header becomes FILLING before any data byte of the slot changes.
-        // In ZEROCOPY mode K1 itself stores into the slot's file pages, so this happens before K1
-        // is launched; otherwise the orchestrator writes it before its first D2H.
+        // In ZEROCOPY mode K1 itself stores into the slot's file pages, and with D2H_UPFRONT the
+        // copies are enqueued with the K1 windows, so this happens before K1 is launched (ADVICE
+        // r01); otherwise the orchestrator writes it before its first D2H.
         int rc = c->engine->filling(ck->t);
         if (rc) fail_ckpt(c, ck, rc);
     }
@@ -669,10 +676,31 @@ void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
     P.tables = c->tables;
     P.consts = c->consts;
     cudaError_t e = cudaSuccess;
-    // publishes a successful window to the orchestrator (a failed one never is)
+    // publishes a successful window to the orchestrator (a failed one never is); with
+    // D2H_UPFRONT this thread enqueues the window's copy-engine D2H itself, right away
+    uint32_t issued = 0;
     auto publish = [&](uint32_t first, uint32_t count) {
         cudaEvent_t ev = get_event(c);
         cudaEventRecord(ev, c->pack_stream);
+        if (c->upfront()) {
+            cudaStreamWaitEvent(c->copy_stream, ev, 0);
+            for (uint32_t j = first; j < first + count;) {
+                const uint64_t r0 = (ck->ring_start + j) % c->ring_slots;
+                uint32_t k = 1;  // chunks contiguous in the ring, up to 64 MiB per copy
+                const uint64_t kmax = std::max<uint64_t>(1, (64ull << 20) / c->cb());
+                while (k < kmax && j + k < first + count && r0 + k < c->ring_slots) ++k;
+                PersistTask task{ck, j, c->map + c->slot_data_off(ck->t.slot) + (uint64_t)j * c->cb(), nullptr, true, k};
+                cudaError_t e2 = cudaMemcpyAsync(task.dest, c->ring + r0 * c->cb(), (uint64_t)k * c->cb(),
+                                                 cudaMemcpyDeviceToHost, c->copy_stream);
+                if (e2 != cudaSuccess) fail_ckpt(c, ck, cuda_error(e2, "D2H"));
+                if (j + k == c->n) cudaEventRecord(ck->ev_landed, c->copy_stream);
+                task.ev = get_event(c);
+                cudaEventRecord(task.ev, c->copy_stream);
+                c->tasks.push(task);
+                j += k;
+                issued = j;
+            }
+        }
         {
             std::lock_guard<std::mutex> lk(ck->mu);
             ck->launches.push_back({first, count, ev});
@@ -727,6 +755,8 @@ void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
             cudaEventRecord(k1e.second, c->pack_stream);
             c->launches += 1;
             if (e != cudaSuccess) break;
+            PCC_TRACE("pack: ckpt %llu window %llu+%llu launched", (unsigned long long)ck->t.counter,
+                      (unsigned long long)done, (unsigned long long)k);
             publish((uint32_t)done, (uint32_t)k);
             done += k;
         }
@@ -769,6 +799,11 @@ void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
         c->packed_seq.store(ck->seq);
     }
     c->pk_cv.notify_all();
+    if (c->upfront()) {  // the orchestrator's end-of-checkpoint accounting, done here
+        const uint32_t unissued = (uint32_t)c->n - issued;
+        for (uint32_t j = issued; j < c->n; ++j) ring_release(c, ck->ring_start + j);  // never issued
+        if (c->n == 0 || (unissued && ck->remaining.fetch_sub(unissued) == unissued)) finish_ckpt(c, ck);
+    }
 }
 
 void pack_loop(pcc_ctx *c) {
@@ -821,6 +856,8 @@ int pcc_open(const pcc_config *cfg, pcc_ctx **out) {
     if ((cfg->flags & PCC_ZEROCOPY) && !(cfg->flags & PCC_MAPFILE))
         return set_error(PCC_EINVAL, "ZEROCOPY needs MAPFILE");
     if (nullsink && (cfg->flags & PCC_MAPFILE)) return set_error(PCC_EINVAL, "NULLSINK excludes MAPFILE");
+    if ((cfg->flags & PCC_D2H_UPFRONT) && !(cfg->flags & PCC_MAPFILE))
+        return set_error(PCC_EINVAL, "D2H_UPFRONT needs MAPFILE (copies straight into the file pages)");
     if ((cfg->allreduce == nullptr) != (cfg->allgather == nullptr))
         return set_error(PCC_EINVAL, "allreduce and allgather callbacks go together");
     if (cfg->world > 1 && !(cfg->flags & PCC_NOCOMM) && !cfg->allreduce && !cfg->nccl_unique_id)
@@ -1053,7 +1090,7 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
         c->ckpts[ck->t.counter] = ck;
     }
     c->guard_armed = true;
-    c->jobs.push(ck);  // the orchestrator follows the K1 windows as they are published
+    if (!c->upfront()) c->jobs.push(ck);  // the orchestrator follows the K1 windows as they are published
     // K1: enqueued right here when nothing is queued ahead of it and the HBM ring already has room
     // for the whole slice (the usual case: the previous checkpoints drained within the interval);
     // otherwise the packer thread launches the windows as ring space frees.  Either way this call
@@ -1063,6 +1100,8 @@ int pcc_checkpoint(pcc_ctx *c, uint64_t iter, void *train_stream, pcc_handle *ou
         std::lock_guard<std::mutex> lk(c->ring_mu);
         inline_pack = c->ring_tail + c->ring_slots >= c->ring_head + c->n;
     }
+    PCC_TRACE("ckpt %llu iter %llu seq %u: %s", (unsigned long long)ck->t.counter, (unsigned long long)iter, ck->seq,
+              inline_pack ? "K1 inline" : "to the packer");
     if (inline_pack) {
         pack_one(c, ck);
     } else {
@@ -1081,8 +1120,10 @@ int pcc_guard(pcc_ctx *c, void *train_stream) {
     // only when the packer thread still holds K1 windows of the newest checkpoint (ring space):
     // wait here, on the host and outside any CUDA call, until they are enqueued
     if ((int32_t)(c->packed_seq.load() - want) < 0) {
+        PCC_TRACE("guard: seq %u waits for the packer", want);
         std::unique_lock<std::mutex> lk(c->pk_mu);
         c->pk_cv.wait(lk, [&] { return (int32_t)(c->packed_seq.load() - want) >= 0; });
+        PCC_TRACE("guard: seq %u released", want);
     }
     cudaError_t e = cudaStreamWaitEvent(ts, c->ev_guard, 0);
     return e == cudaSuccess ? PCC_OK : cuda_error(e, "guard");

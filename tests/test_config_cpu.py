@@ -12,6 +12,8 @@ pcc = pytest.importorskip("paper_conf_asplos_strati0k25_b200")
     dict(max_inflight=0),
     dict(flags=pcc.ZEROCOPY),                                # Variant A needs the file mapping
     dict(flags=pcc.NULLSINK | pcc.MAPFILE),
+    dict(flags=pcc.D2H_UPFRONT),                             # upfront copies go straight into the mapping
+    dict(flags=pcc.NULLSINK | pcc.D2H_UPFRONT),
     dict(rank=2, world=2),
     dict(world=0),
     dict(world=2),                                           # no NCCL id and no callbacks

@@ -66,7 +66,7 @@ def run_protocol(ck, stream, fwd_bwd, update, every=10, iters=200, warmup=20, ru
     per-position extra ms, the host time of every pcc_checkpoint call, the drain times and the
     contended snapshot rate)."""
     import torch
-    host_ms, infos, drain_ms = [], [], []
+    host_ms, infos, drain_ms, guard_ms = [], [], [], []
 
     def loop(n, checkpoint, it0):
         evs = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
@@ -77,7 +77,10 @@ def run_protocol(ck, stream, fwd_bwd, update, every=10, iters=200, warmup=20, ru
                 evs[i - host_lead].synchronize()
             fwd_bwd()
             if checkpoint and use_guard:
+                tg = time.perf_counter()
                 ck.guard(stream)
+                if i % every == 1 and i > 1:
+                    guard_ms.append((time.perf_counter() - tg) * 1e3)
             update()
             if checkpoint and i % every == 0:
                 th = time.perf_counter()
@@ -101,6 +104,7 @@ def run_protocol(ck, stream, fwd_bwd, update, every=10, iters=200, warmup=20, ru
     host_ms.clear()
     infos.clear()
     drain_ms.clear()
+    guard_ms.clear()
     base_t, ck_t, its_b, its_c = [], [], [], []
     pos_b, pos_c = [[] for _ in range(every)], [[] for _ in range(every)]
     it0 = 1000
@@ -129,7 +133,12 @@ def run_protocol(ck, stream, fwd_bwd, update, every=10, iters=200, warmup=20, ru
         "extra_ms_by_pos": [statistics.mean(pc) - statistics.mean(pb) for pb, pc in zip(pos_b, pos_c)],
         "host_ckpt_call_ms": statistics.median(host_ms) if host_ms else None,
         "host_ckpt_call_ms_max": max(host_ms) if host_ms else None,
+        # the U-gate call right after a checkpoint: host time (it waits only while the packer
+        # thread still holds K1 windows of that checkpoint, i.e. the HBM ring was full)
+        "host_guard_ms": statistics.median(guard_ms) if guard_ms else None,
+        "host_guard_ms_max": max(guard_ms) if guard_ms else None,
         "drain_ms": statistics.median(drain_ms) if drain_ms else None,
+        "iters_ms_ckpt_last_run": [round(x, 2) for x in its_c[-iters:]],
         "contended": None if not infos else {
             "checkpoints": len(infos), "k1_busy_ms": statistics.median(i["k1_busy_ms"] for i in infos),
             "pack_span_ms": statistics.median(i["pack_ms"] for i in infos), "snapshot_ms": snap,
@@ -140,13 +149,13 @@ def run_protocol(ck, stream, fwd_bwd, update, every=10, iters=200, warmup=20, ru
 
 
 def _open(pcc, state, path, chunk_bytes, n_inflight, flags, d2h_gbs, d2h_quantum, dev, rank=0, world=1,
-          ck_kwargs=None, ring_bytes=0):
+          ck_kwargs=None, ring_bytes=0, pack_ctas=0):
     shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
     path = path or os.path.join(shm, f"pcc_slowdown_{os.getpid()}_{time.monotonic_ns()}.pcc")
     ck = pcc.PCCheck(None if flags == pcc.NULLSINK else path, chunk_bytes=chunk_bytes, max_inflight=n_inflight,
                      flags=pcc.MAPFILE if flags is None else flags, ring_bytes=ring_bytes,
                      staging_bytes=8 * chunk_bytes, d2h_gbs=d2h_gbs or 0.0, d2h_quantum=d2h_quantum or 0,
-                     device=dev, rank=rank, world=world, **(ck_kwargs or {}))
+                     device=dev, rank=rank, world=world, pack_ctas=pack_ctas, **(ck_kwargs or {}))
     ck.register(state)
     return ck, path
 
@@ -222,6 +231,8 @@ def vgg16_slowdown(pcc, iters=200, every=10, warmup=20, batch=32, runs=3, path=N
     if d2h_gbs == "auto":
         d2h_gbs, d2h_quantum, pace_choice = _auto_pace(pcc, state, chunk_bytes, every, link_gbs,
                                                        lambda: (fwd_bwd(), update()), stream, rank, world)
+    if flags is None and graphs:  # a CUDA-graph loop: the D2H is enqueued with K1 (PCC_D2H_UPFRONT)
+        flags, d2h_gbs, d2h_quantum = pcc.MAPFILE | pcc.D2H_UPFRONT, 0.0, 0
     ck, path = _open(pcc, state, path, chunk_bytes, n_inflight, flags, d2h_gbs, d2h_quantum, dev.index, rank, world,
                      ck_kwargs)
     nbytes = sum(t.numel() * t.element_size() for t in state)
@@ -237,7 +248,7 @@ def vgg16_slowdown(pcc, iters=200, every=10, warmup=20, batch=32, runs=3, path=N
 
 def hf_slowdown(pcc, model="bert", iters=200, every=10, warmup=20, runs=3, path=None, n_inflight=2,
                 chunk_bytes=64 << 20, d2h_gbs=0.0, d2h_quantum=0, link_gbs=None, flags=None, ring_bytes=0,
-                use_guard=True, graphs=False, host_lead=None):
+                use_guard=True, graphs=False, host_lead=None, pack_ctas=0):
     """model="bert": BERT-large QA (24 layers, hidden 1024), fp32, batch 3 x 384 tokens, Adam(fused);
     model="opt13": OPT-1.3B, fp32 params, Adam(fused), bf16 autocast, batch 1 x 2048 tokens.
     The checkpointed state is R11's registration of the optimizer (param, exp_avg, exp_avg_sq,
@@ -293,15 +304,18 @@ def hf_slowdown(pcc, model="bert", iters=200, every=10, warmup=20, runs=3, path=
     if d2h_gbs == "auto":
         d2h_gbs, d2h_quantum, pace_choice = _auto_pace(pcc, state, chunk_bytes, every, link_gbs,
                                                        lambda: (fwd_bwd(), update()), stream)
+    if flags is None and graphs:  # a CUDA-graph loop: the D2H is enqueued with K1 (PCC_D2H_UPFRONT)
+        flags, d2h_gbs, d2h_quantum = pcc.MAPFILE | pcc.D2H_UPFRONT, 0.0, 0
     ck, path = _open(pcc, state, path, chunk_bytes, n_inflight, flags, d2h_gbs, d2h_quantum, dev.index,
-                     ring_bytes=ring_bytes)
+                     ring_bytes=ring_bytes, pack_ctas=pack_ctas)
     nbytes = sum(t.numel() * t.element_size() for t in state)
     res = run_protocol(ck, stream, fwd_bwd, update, every, iters, warmup, runs, host_lead, use_guard, False, nbytes)
     return _finish(ck, path, res, model=desc + ", random init, synthetic inputs"
                    + (", step as 2 CUDA graphs (fwd+bwd | optimizer)" if graphs else ", eager"),
                    N=n_inflight, graphs=graphs, guard=use_guard, d2h_gbs=d2h_gbs or None,
                    d2h_quantum=d2h_quantum or None, pace_choice=pace_choice, state_bytes=nbytes, tensors=len(state),
-                   ring_bytes=ring_bytes or None)
+                   ring_bytes=ring_bytes or None, d2h_upfront=bool(flags and flags & pcc.D2H_UPFRONT),
+                   pack_ctas=pack_ctas or None)
 
 
 def bloom_slowdown(pcc, world=8, iters=200, every=10, warmup=20, runs=3, seq=2048, path=None, d2h_gbs=0.0,
@@ -379,6 +393,9 @@ if __name__ == "__main__":
     ap.add_argument("--every", type=int, default=10)
     ap.add_argument("--host-lead", type=int, default=0)
     ap.add_argument("--link-gbs", type=float, default=55.0)
+    ap.add_argument("--inflight", type=int, default=2)
+    ap.add_argument("--pack-ctas", type=int, default=0)
+    ap.add_argument("--ring-slices", type=float, default=0, help="HBM ring in slices (0 = one slice)")
     a = ap.parse_args()
     import paper_conf_asplos_strati0k25_b200 as pcc
     pace = a.pace if a.pace == "auto" else float(a.pace)
@@ -388,5 +405,11 @@ if __name__ == "__main__":
     elif a.model == "bloom":
         r = bloom_slowdown(pcc, **kw)
     else:
-        r = hf_slowdown(pcc, a.model, graphs=a.graphs, host_lead=a.host_lead or None, **kw)
+        ring = 0
+        if a.ring_slices:
+            from synth import config_tensors
+            nb = sum(t.nbytes for t in config_tensors({"opt13": "c3", "bert": "bert"}[a.model]))
+            ring = int(a.ring_slices * -(-nb // (64 << 20))) * (64 << 20)
+        r = hf_slowdown(pcc, a.model, graphs=a.graphs, host_lead=a.host_lead or None, n_inflight=a.inflight,
+                        ring_bytes=ring, pack_ctas=a.pack_ctas, **kw)
     print(json.dumps(r))
