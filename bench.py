@@ -316,13 +316,17 @@ def run_slowdowns(args, pcc, rank, world, coll, uid, peak_link, emu, torch, dist
                     return S.vgg16_slowdown(pcc, rank=rank, world=world, ck_kwargs=ckw, **kw, **extra)
                 plans.append((name, fn))
         else:
-            plans = [("slowdown", lambda: S.vgg16_slowdown(pcc, graphs=True, **kw, **auto)),
+            plans = [("slowdown", lambda: S.vgg16_slowdown(pcc, graphs=True, host_lead=2, **kw, **auto)),
                      ("slowdown_eager", lambda: S.vgg16_slowdown(pcc, **kw, **auto)),
                      ("slowdown_unpaced", lambda: S.vgg16_slowdown(pcc, **kw))]
     elif args.config == "c3" and world == 1:
-        plans = [("slowdown", lambda: S.hf_slowdown(pcc, "opt13", graphs=True, n_inflight=args.inflight, **kw, **auto)),
-                 ("slowdown_eager", lambda: S.hf_slowdown(pcc, "opt13", n_inflight=args.inflight, **kw, **auto)),
-                 ("slowdown_unpaced", lambda: S.hf_slowdown(pcc, "opt13", n_inflight=args.inflight, **kw))]
+        o = dict(n_inflight=args.inflight, **kw)
+        plans = [  # graphs + the tuner's graph pace, host <= 2 replays ahead (a loop that reads its loss)
+                 ("slowdown", lambda: S.hf_slowdown(pcc, "opt13", graphs=True, host_lead=2, **o, **auto)),
+                 # graphs, host unthrottled (runs into a full launch queue): PCC_D2H_UPFRONT, unpaced
+                 ("slowdown_graphs_unthrottled", lambda: S.hf_slowdown(pcc, "opt13", graphs=True, **o)),
+                 ("slowdown_eager", lambda: S.hf_slowdown(pcc, "opt13", **o, **auto)),
+                 ("slowdown_unpaced", lambda: S.hf_slowdown(pcc, "opt13", **o))]
     elif args.config == "bert" and world == 1:
         plans = [("slowdown", lambda: S.hf_slowdown(pcc, "bert", **kw, **auto)),
                  ("slowdown_unpaced", lambda: S.hf_slowdown(pcc, "bert", **kw))]
@@ -561,8 +565,9 @@ def main():
     # training slowdown, checkpoint every 10 iterations (BASELINE metric, second half), on the
     # config's own model with SURVEY §8(d)'s protocol (tools/slowdown.run_protocol: 20 warm-up +
     # --slowdown-iters x --slowdown-runs, p50/p99, final drain):
-    #   slowdown           the library as configured for training: the tuner's D2H pace
-    #                      (tuner.choose_pace) — OPT-1.3B / VGG-16: step as 2 CUDA graphs
+    #   slowdown           the library as configured for training: the step as 2 CUDA graphs, the
+    #                      tuner's graph D2H pace (tuner.choose_pace), host <= 2 replays ahead
+    #   slowdown_graphs_unthrottled  (C3) graphs with the host unthrottled: PCC_D2H_UPFRONT
     #   slowdown_eager     eager PyTorch, tuned pace
     #   slowdown_unpaced   eager PyTorch, unpaced (the transfer configuration `value` is measured in)
     #   world > 1: DDP on every rank, each checkpointing its 1/world slice with the collective

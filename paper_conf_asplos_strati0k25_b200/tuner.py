@@ -85,9 +85,20 @@ def tune(make_ctx, m_bytes: int, S_bytes: int, t: float, q: float, n_max: int = 
 D2H_QUANTUM = 512 << 10  # bytes per paced copy (0.5 MiB: measured best trade, r01 diagnosis)
 
 
+GRAPH_MARGIN = 0.8   # a CUDA-graph training loop: land a checkpoint within 0.8 of its interval
+GRAPH_QUANTUM = 4 << 20
+
+
 def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, margin: float = 0.5,
-                max_margin: float = 0.5, n_inflight: int = 2) -> dict:
+                max_margin: float = 0.5, n_inflight: int = 2, graphs: bool = False) -> dict:
     """D2H pace for training: {"d2h_gbs": G, "d2h_quantum": Q}; G = 0 means unpaced.
+
+    graphs=True (the training step replayed as CUDA graphs): the gentlest pace that lands one
+    checkpoint within GRAPH_MARGIN of its interval, in GRAPH_QUANTUM copies.  Measured on
+    OPT-1.3B (15.8 GB every 10 x 51.7 ms, profiles/r02_graph_pace.jsonl): unpaced 3.8%, 40 GB/s
+    (lands at 0.82 of the interval) 1.4%, 30 GB/s (1.0: the next K1 overlaps the tail) 1.9-2.3%:
+    a graph replay pays per byte in flight on the link, so a longer, gentler transfer is cheaper,
+    unlike the eager loop below whose cost per byte moved stays constant.
 
     The gentlest pace that lands one checkpoint within `margin` of its interval f*t, never below
     half the link (below that the measured cost no longer drops).  When that needs more than
@@ -98,6 +109,12 @@ def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, margin: flo
     unpaced — there the answer is a longer interval (Eq 3's f*), not a pace."""
     if f <= 0 or t <= 0 or link_gbs <= 0:
         raise ValueError("f, t and link_gbs must be positive")
+    if graphs:
+        need = slice_bytes / (GRAPH_MARGIN * f * t) / 1e9
+        g = max(need, 0.5 * link_gbs)
+        if g >= link_gbs:
+            return {"d2h_gbs": 0.0, "d2h_quantum": 0, "need_gbs": need}
+        return {"d2h_gbs": g, "d2h_quantum": GRAPH_QUANTUM, "need_gbs": need}
     need = slice_bytes / (margin * f * t) / 1e9  # GB/s to land a checkpoint in margin * f * t
     g = max(need, 0.5 * link_gbs)
     if g >= link_gbs and n_inflight >= 2 and max_margin > margin:

@@ -45,10 +45,10 @@ def _slice_bytes(pcc, state, chunk_bytes, rank=0, world=1):
     return (((rank + 1) * c) // world - (rank * c) // world) * chunk_bytes
 
 
-def _auto_pace(pcc, state, chunk_bytes, every, link_gbs, step_fn, stream, rank=0, world=1):
+def _auto_pace(pcc, state, chunk_bytes, every, link_gbs, step_fn, stream, rank=0, world=1, graphs=False):
     from paper_conf_asplos_strati0k25_b200.tuner import choose_pace
     t = _iter_time(step_fn, stream)
-    choice = choose_pace(_slice_bytes(pcc, state, chunk_bytes, rank, world), every, t, link_gbs)
+    choice = choose_pace(_slice_bytes(pcc, state, chunk_bytes, rank, world), every, t, link_gbs, graphs=graphs)
     choice.update(t_iter_s=t, link_gbs=link_gbs)
     return choice["d2h_gbs"], choice["d2h_quantum"], choice
 
@@ -230,9 +230,9 @@ def vgg16_slowdown(pcc, iters=200, every=10, warmup=20, batch=32, runs=3, path=N
     pace_choice = None
     if d2h_gbs == "auto":
         d2h_gbs, d2h_quantum, pace_choice = _auto_pace(pcc, state, chunk_bytes, every, link_gbs,
-                                                       lambda: (fwd_bwd(), update()), stream, rank, world)
-    if flags is None and graphs:  # a CUDA-graph loop: the D2H is enqueued with K1 (PCC_D2H_UPFRONT)
-        flags, d2h_gbs, d2h_quantum = pcc.MAPFILE | pcc.D2H_UPFRONT, 0.0, 0
+                                                       lambda: (fwd_bwd(), update()), stream, rank, world, graphs)
+    if flags is None and graphs and not d2h_gbs:  # an unpaced CUDA-graph loop: PCC_D2H_UPFRONT
+        flags = pcc.MAPFILE | pcc.D2H_UPFRONT
     ck, path = _open(pcc, state, path, chunk_bytes, n_inflight, flags, d2h_gbs, d2h_quantum, dev.index, rank, world,
                      ck_kwargs)
     nbytes = sum(t.numel() * t.element_size() for t in state)
@@ -248,7 +248,7 @@ def vgg16_slowdown(pcc, iters=200, every=10, warmup=20, batch=32, runs=3, path=N
 
 def hf_slowdown(pcc, model="bert", iters=200, every=10, warmup=20, runs=3, path=None, n_inflight=2,
                 chunk_bytes=64 << 20, d2h_gbs=0.0, d2h_quantum=0, link_gbs=None, flags=None, ring_bytes=0,
-                use_guard=True, graphs=False, host_lead=None, pack_ctas=0):
+                use_guard=True, graphs=False, host_lead=None, pack_ctas=0, upfront=None):
     """model="bert": BERT-large QA (24 layers, hidden 1024), fp32, batch 3 x 384 tokens, Adam(fused);
     model="opt13": OPT-1.3B, fp32 params, Adam(fused), bf16 autocast, batch 1 x 2048 tokens.
     The checkpointed state is R11's registration of the optimizer (param, exp_avg, exp_avg_sq,
@@ -303,8 +303,10 @@ def hf_slowdown(pcc, model="bert", iters=200, every=10, warmup=20, runs=3, path=
     pace_choice = None
     if d2h_gbs == "auto":
         d2h_gbs, d2h_quantum, pace_choice = _auto_pace(pcc, state, chunk_bytes, every, link_gbs,
-                                                       lambda: (fwd_bwd(), update()), stream)
-    if flags is None and graphs:  # a CUDA-graph loop: the D2H is enqueued with K1 (PCC_D2H_UPFRONT)
+                                                       lambda: (fwd_bwd(), update()), stream, graphs=graphs)
+    if upfront is None:  # default: an unpaced CUDA-graph loop enqueues the D2H with K1
+        upfront = graphs and not d2h_gbs
+    if flags is None and upfront:  # PCC_D2H_UPFRONT (unpaced by construction)
         flags, d2h_gbs, d2h_quantum = pcc.MAPFILE | pcc.D2H_UPFRONT, 0.0, 0
     ck, path = _open(pcc, state, path, chunk_bytes, n_inflight, flags, d2h_gbs, d2h_quantum, dev.index,
                      ring_bytes=ring_bytes, pack_ctas=pack_ctas)
@@ -395,6 +397,8 @@ if __name__ == "__main__":
     ap.add_argument("--link-gbs", type=float, default=55.0)
     ap.add_argument("--inflight", type=int, default=2)
     ap.add_argument("--pack-ctas", type=int, default=0)
+    ap.add_argument("--no-upfront", action="store_true", help="graphs: keep the orchestrator-issued (pace-able) D2H")
+    ap.add_argument("--quantum-kib", type=int, default=512)
     ap.add_argument("--ring-slices", type=float, default=0, help="HBM ring in slices (0 = one slice)")
     a = ap.parse_args()
     import paper_conf_asplos_strati0k25_b200 as pcc
@@ -411,5 +415,6 @@ if __name__ == "__main__":
             nb = sum(t.nbytes for t in config_tensors({"opt13": "c3", "bert": "bert"}[a.model]))
             ring = int(a.ring_slices * -(-nb // (64 << 20))) * (64 << 20)
         r = hf_slowdown(pcc, a.model, graphs=a.graphs, host_lead=a.host_lead or None, n_inflight=a.inflight,
-                        ring_bytes=ring, pack_ctas=a.pack_ctas, **kw)
+                        ring_bytes=ring, pack_ctas=a.pack_ctas, upfront=False if a.no_upfront else None,
+                        d2h_quantum=(a.quantum_kib << 10) if pace else 0, **kw)
     print(json.dumps(r))
