@@ -319,6 +319,17 @@ def run_slowdowns(args, pcc, rank, world, coll, uid, peak_link, emu, torch, dist
             plans = [("slowdown", lambda: S.vgg16_slowdown(pcc, graphs=True, host_lead=2, **kw, **auto)),
                      ("slowdown_eager", lambda: S.vgg16_slowdown(pcc, **kw, **auto)),
                      ("slowdown_unpaced", lambda: S.vgg16_slowdown(pcc, **kw))]
+    elif args.config == "c3" and world > 1:  # OPT-1.3B under DDP, every rank its 1/world slice
+        ckw = dict(coll) if coll else {"nccl_unique_id": None}
+        for name, extra in (("slowdown", auto), ("slowdown_unpaced", {})):
+            def fn(extra=extra):
+                if not coll:
+                    obj = [pcc.nccl_unique_id() if rank == 0 else None]
+                    dist.broadcast_object_list(obj, src=0)
+                    ckw["nccl_unique_id"] = obj[0]
+                return S.hf_slowdown(pcc, "opt13", n_inflight=args.inflight, rank=rank, world=world, ck_kwargs=ckw,
+                                     **kw, **extra)
+            plans.append((name, fn))
     elif args.config == "c3" and world == 1:
         o = dict(n_inflight=args.inflight, **kw)
         plans = [  # graphs + the tuner's graph pace, host <= 2 replays ahead (a loop that reads its loss)
@@ -584,7 +595,7 @@ def main():
     if rank == 0:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
             peaks = json.load(f)
-        k1_bytes = 2 * slice_bytes  # read the slice's state bytes + write the packed slice (R3: pads count)
+        k1_bytes = rank_state_bytes + slice_bytes  # read the slice's state bytes + write the packed slice (R3: pads count)
         k1_achieved = k1_bytes / (k1_ms * 1e-3) / 1e9
         link_achieved = slice_bytes / (ms_total * 1e-3 / args.steps) / 1e9
         line = {

@@ -86,7 +86,7 @@ D2H_QUANTUM = 512 << 10  # bytes per paced copy (0.5 MiB: measured best trade, r
 
 
 GRAPH_MARGIN = 0.8   # a CUDA-graph training loop: land a checkpoint within 0.8 of its interval
-GRAPH_QUANTUM = 4 << 20
+GRAPH_QUANTUM = 1 << 20  # 1 MiB copies: 4 MiB ones cost ~3x more per burst iteration (r02_graph_pace_quantum)
 
 
 def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, margin: float = 0.5,
@@ -94,11 +94,13 @@ def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, margin: flo
     """D2H pace for training: {"d2h_gbs": G, "d2h_quantum": Q}; G = 0 means unpaced.
 
     graphs=True (the training step replayed as CUDA graphs): the gentlest pace that lands one
-    checkpoint within GRAPH_MARGIN of its interval, in GRAPH_QUANTUM copies.  Measured on
-    OPT-1.3B (15.8 GB every 10 x 51.7 ms, profiles/r02_graph_pace.jsonl): unpaced 3.8%, 40 GB/s
-    (lands at 0.82 of the interval) 1.4%, 30 GB/s (1.0: the next K1 overlaps the tail) 1.9-2.3%:
-    a graph replay pays per byte in flight on the link, so a longer, gentler transfer is cheaper,
-    unlike the eager loop below whose cost per byte moved stays constant.
+    checkpoint within GRAPH_MARGIN of its interval, in GRAPH_QUANTUM copies.  Measured on one box,
+    OPT-1.3B (15.8 GB every 10 x 51.7 ms, 200 iterations each, profiles/r02_graph_pace_quantum.jsonl):
+    unpaced 3.9%; 35 / 40 / 45 GB/s in 1 MiB copies 1.1 / - / 1.8%, in 0.5 MiB 1.7 / 1.4 / 1.6% (at
+    45 GB/s the host no longer keeps a 12 us cadence: 0.83 of the pace delivered), in 4 MiB 3.3 /
+    - / 3.0%.  A graph replay pays per byte in flight on the link, so a longer, gentler transfer
+    in small copies is cheaper — unlike the eager loop below, whose cost per byte moved stays
+    constant whatever the pace.
 
     The gentlest pace that lands one checkpoint within `margin` of its interval f*t, never below
     half the link (below that the measured cost no longer drops).  When that needs more than

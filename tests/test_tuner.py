@@ -37,7 +37,7 @@ def test_choose_pace():
     assert choose_pace(15_789_098_512, 10, 0.0438, 57.0, max_margin=0.9, n_inflight=1)["d2h_gbs"] == 0.0
     with pytest.raises(ValueError):
         choose_pace(1, 0, 1.0, 1.0)
-    # a CUDA-graph loop: land within 0.8 of the interval, 4 MiB copies (OPT-1.3B -> ~38 GB/s)
+    # a CUDA-graph loop: land within 0.8 of the interval, 1 MiB copies (OPT-1.3B -> ~38 GB/s)
     from paper_conf_asplos_strati0k25_b200.tuner import GRAPH_QUANTUM
     p = choose_pace(15_789_098_512, 10, 0.0517, 56.7, graphs=True)
     assert p["d2h_gbs"] == pytest.approx(15_789_098_512 / (0.8 * 10 * 0.0517) / 1e9) and p["d2h_quantum"] == GRAPH_QUANTUM

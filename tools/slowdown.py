@@ -248,7 +248,8 @@ def vgg16_slowdown(pcc, iters=200, every=10, warmup=20, batch=32, runs=3, path=N
 
 def hf_slowdown(pcc, model="bert", iters=200, every=10, warmup=20, runs=3, path=None, n_inflight=2,
                 chunk_bytes=64 << 20, d2h_gbs=0.0, d2h_quantum=0, link_gbs=None, flags=None, ring_bytes=0,
-                use_guard=True, graphs=False, host_lead=None, pack_ctas=0, upfront=None):
+                use_guard=True, graphs=False, host_lead=None, pack_ctas=0, upfront=None, rank=0, world=1,
+                ck_kwargs=None):
     """model="bert": BERT-large QA (24 layers, hidden 1024), fp32, batch 3 x 384 tokens, Adam(fused);
     model="opt13": OPT-1.3B, fp32 params, Adam(fused), bf16 autocast, batch 1 x 2048 tokens.
     The checkpointed state is R11's registration of the optimizer (param, exp_avg, exp_avg_sq,
@@ -267,7 +268,7 @@ def hf_slowdown(pcc, model="bert", iters=200, every=10, warmup=20, runs=3, path=
         ends = torch.randint(0, 384, (3,), device=dev)
 
         def loss_fn():
-            return net(input_ids=ids, start_positions=starts, end_positions=ends).loss
+            return model_fwd(input_ids=ids, start_positions=starts, end_positions=ends).loss
         desc = "BERT-large QA fp32, Adam(fused), batch 3 x 384 tokens"
     elif model == "opt13":
         from transformers import OPTConfig, OPTForCausalLM
@@ -281,12 +282,19 @@ def hf_slowdown(pcc, model="bert", iters=200, every=10, warmup=20, runs=3, path=
 
         def loss_fn():
             with torch.autocast("cuda", dtype=torch.bfloat16, cache_enabled=not graphs):
-                return net(input_ids=ids, attention_mask=mask if graphs else None, labels=ids).loss
+                return model_fwd(input_ids=ids, attention_mask=mask if graphs else None, labels=ids).loss
         desc = "OPT-1.3B fp32 params, Adam(fused), bf16 autocast, batch 1 x 2048 tokens"
     else:
         raise ValueError(model)
     net.train()
     opt = torch.optim.Adam(net.parameters(), lr=1e-5, fused=True, capturable=graphs)
+    if world > 1:  # data parallelism: DDP allreduces the gradients, the state stays replicated
+        if graphs:
+            raise ValueError("world > 1 runs eager (DDP)")
+        ddp = torch.nn.parallel.DistributedDataParallel(net, device_ids=[dev.index])
+        model_fwd = ddp
+    else:
+        model_fwd = net
     stream = torch.cuda.current_stream()
 
     def fwd_bwd():
@@ -303,17 +311,19 @@ def hf_slowdown(pcc, model="bert", iters=200, every=10, warmup=20, runs=3, path=
     pace_choice = None
     if d2h_gbs == "auto":
         d2h_gbs, d2h_quantum, pace_choice = _auto_pace(pcc, state, chunk_bytes, every, link_gbs,
-                                                       lambda: (fwd_bwd(), update()), stream, graphs=graphs)
+                                                       lambda: (fwd_bwd(), update()), stream, rank, world, graphs)
     if upfront is None:  # default: an unpaced CUDA-graph loop enqueues the D2H with K1
         upfront = graphs and not d2h_gbs
     if flags is None and upfront:  # PCC_D2H_UPFRONT (unpaced by construction)
         flags, d2h_gbs, d2h_quantum = pcc.MAPFILE | pcc.D2H_UPFRONT, 0.0, 0
-    ck, path = _open(pcc, state, path, chunk_bytes, n_inflight, flags, d2h_gbs, d2h_quantum, dev.index,
-                     ring_bytes=ring_bytes, pack_ctas=pack_ctas)
+    ck, path = _open(pcc, state, path, chunk_bytes, n_inflight, flags, d2h_gbs, d2h_quantum, dev.index, rank, world,
+                     ck_kwargs, ring_bytes=ring_bytes, pack_ctas=pack_ctas)
     nbytes = sum(t.numel() * t.element_size() for t in state)
-    res = run_protocol(ck, stream, fwd_bwd, update, every, iters, warmup, runs, host_lead, use_guard, False, nbytes)
+    res = run_protocol(ck, stream, fwd_bwd, update, every, iters, warmup, runs, host_lead, use_guard, world > 1,
+                       nbytes if world == 1 else _slice_bytes(pcc, state, chunk_bytes, rank, world))
     return _finish(ck, path, res, model=desc + ", random init, synthetic inputs"
-                   + (", step as 2 CUDA graphs (fwd+bwd | optimizer)" if graphs else ", eager"),
+                   + (", step as 2 CUDA graphs (fwd+bwd | optimizer)" if graphs else ", eager")
+                   + (f", DDP over {world} ranks (this rank: {rank}; its 1/{world} slice)" if world > 1 else ""),
                    N=n_inflight, graphs=graphs, guard=use_guard, d2h_gbs=d2h_gbs or None,
                    d2h_quantum=d2h_quantum or None, pace_choice=pace_choice, state_bytes=nbytes, tensors=len(state),
                    ring_bytes=ring_bytes or None, d2h_upfront=bool(flags and flags & pcc.D2H_UPFRONT),
