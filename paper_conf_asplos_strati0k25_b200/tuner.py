@@ -11,11 +11,9 @@ Here T_w of one checkpoint is measured by the library itself (pcc_info: pcc_chec
 -> local commit) while N checkpoints are kept in flight at a cadence of one every t seconds.
 
 On B200 the tool also picks the D2H pace (pcc_config d2h_mbps / d2h_quantum): a saturating
-copy-engine burst slows an eager training loop by ~10% while it lasts, small paced copies
-leave gaps that hide it (profiles/r01_slowdown_diagnosis.md).  `choose_pace` takes the
-gentlest pace that still lands one checkpoint within `margin` of its interval f*t, never below
-half the link (below that the measured interference no longer drops) and unpaced when even the
-full link is needed.
+copy-engine burst slows a training loop while it lasts, and small paced copies hide most of it
+(`choose_pace`, measured rule in its docstring).  It also picks the buffer size b from T_G
+(`choose_chunk`, L176) and where K1 puts the chunks under an HBM budget (`choose_ring`).
 """
 from __future__ import annotations
 
@@ -82,46 +80,40 @@ def tune(make_ctx, m_bytes: int, S_bytes: int, t: float, q: float, n_max: int = 
     return out
 
 
-D2H_QUANTUM = 512 << 10  # bytes per paced copy (0.5 MiB: measured best trade, r01 diagnosis)
+D2H_QUANTUM = 1 << 20    # bytes per paced copy (1 MiB: r02 sweeps, eager and graphs)
+EAGER_MARGIN, EAGER_CAP = 0.9, 0.7   # eager loop: land within 0.9 of the interval, pace <= 0.7 x link
+GRAPH_MARGIN, GRAPH_CAP = 0.85, 0.85  # CUDA-graph loop
+GRAPH_QUANTUM = D2H_QUANTUM
 
 
-GRAPH_MARGIN = 0.8   # a CUDA-graph training loop: land a checkpoint within 0.8 of its interval
-GRAPH_QUANTUM = 1 << 20  # 1 MiB copies: 4 MiB ones cost ~3x more per burst iteration (r02_graph_pace_quantum)
+def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, n_inflight: int = 2,
+                graphs: bool = False) -> dict:
+    """D2H pace for training: {"d2h_gbs": G, "d2h_quantum": Q, "need_gbs": ...}; G = 0 = unpaced.
 
+    The gentlest pace that lands one checkpoint within a margin of its interval f*t, never below
+    half the link, in 1 MiB copies; unpaced when that needs more than a cap of the link.  The
+    rule is the measured one (round 2, after the pacer was fixed to deliver its rate — the
+    round-1 sweeps ran at ~1/3 of their nominal pace):
 
-def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, margin: float = 0.5,
-                max_margin: float = 0.5, n_inflight: int = 2, graphs: bool = False) -> dict:
-    """D2H pace for training: {"d2h_gbs": G, "d2h_quantum": Q}; G = 0 means unpaced.
-
-    graphs=True (the training step replayed as CUDA graphs): the gentlest pace that lands one
-    checkpoint within GRAPH_MARGIN of its interval, in GRAPH_QUANTUM copies.  Measured on one box,
-    OPT-1.3B (15.8 GB every 10 x 51.7 ms, 200 iterations each, profiles/r02_graph_pace_quantum.jsonl):
-    unpaced 3.9%; 35 / 40 / 45 GB/s in 1 MiB copies 1.1 / - / 1.8%, in 0.5 MiB 1.7 / 1.4 / 1.6% (at
-    45 GB/s the host no longer keeps a 12 us cadence: 0.83 of the pace delivered), in 4 MiB 3.3 /
-    - / 3.0%.  A graph replay pays per byte in flight on the link, so a longer, gentler transfer
-    in small copies is cheaper — unlike the eager loop below, whose cost per byte moved stays
-    constant whatever the pace.
-
-    The gentlest pace that lands one checkpoint within `margin` of its interval f*t, never below
-    half the link (below that the measured cost no longer drops).  When that needs more than
-    the link and N >= 2 checkpoints may overlap (Fig 6), the interval may be
-    stretched up to `max_margin` before giving up the pace.  Off by default (max_margin =
-    margin): measured on OPT-1.3B (15.8 GB every 10 x 44 ms: 72 GB/s at margin 0.5, 40 GB/s at
-    0.9) the stretched pace kept the link busy the whole interval and cost 19.8% against 16.7%
-    unpaced — there the answer is a longer interval (Eq 3's f*), not a pace."""
+    * CUDA-graph loop (OPT-1.3B, 15.8 GB every 10 x 51.7 ms, profiles/r02_graph_pace_quantum.jsonl):
+      unpaced 3.9%; 35 / 45 GB/s in 1 MiB copies 1.1 / 1.8%; 4 MiB copies 3.0-3.3%.  A replay pays
+      per byte in flight on the link, so a long gentle transfer in small copies is cheap:
+      margin 0.85, cap 0.85 of the link.
+    * eager loop (OPT-1.3B, 10 x 44 ms, profiles/r02_eager_pace.jsonl): unpaced 18.9%; 40 GB/s in
+      1 MiB copies 6.5%; 50 GB/s 63% — near the link the copy queue never runs dry and the
+      training's own small D2H (HF's per-forward flag read) waits behind it (the r01 starvation);
+      256 KiB copies: the host cannot keep the cadence (0.57 of the pace delivered).  Margin 0.9,
+      cap 0.7 of the link.
+    n_inflight: a pace that lands after 0.5 of the interval overlaps the next checkpoint's K1 only
+    when N >= 2 lets it start (the bench and the harness run N >= 2)."""
     if f <= 0 or t <= 0 or link_gbs <= 0:
         raise ValueError("f, t and link_gbs must be positive")
-    if graphs:
-        need = slice_bytes / (GRAPH_MARGIN * f * t) / 1e9
-        g = max(need, 0.5 * link_gbs)
-        if g >= link_gbs:
-            return {"d2h_gbs": 0.0, "d2h_quantum": 0, "need_gbs": need}
-        return {"d2h_gbs": g, "d2h_quantum": GRAPH_QUANTUM, "need_gbs": need}
+    margin, cap = (GRAPH_MARGIN, GRAPH_CAP) if graphs else (EAGER_MARGIN, EAGER_CAP)
+    if n_inflight < 2:
+        margin = min(margin, 0.5)
     need = slice_bytes / (margin * f * t) / 1e9  # GB/s to land a checkpoint in margin * f * t
     g = max(need, 0.5 * link_gbs)
-    if g >= link_gbs and n_inflight >= 2 and max_margin > margin:
-        g = max(slice_bytes / (max_margin * f * t) / 1e9, 0.5 * link_gbs)
-    if g >= link_gbs:
+    if g > cap * link_gbs:
         return {"d2h_gbs": 0.0, "d2h_quantum": 0, "need_gbs": need}
     return {"d2h_gbs": g, "d2h_quantum": D2H_QUANTUM, "need_gbs": need}
 

@@ -18,30 +18,29 @@ def test_choose_matches_eq3():
 
 def test_choose_pace():
     from paper_conf_asplos_strati0k25_b200.tuner import D2H_QUANTUM, choose_pace
-    # VGG-16: 1.1 GB every 10 x 17 ms needs 12.9 GB/s at margin 0.5 -> floor of half the link
+    # VGG-16: 1.1 GB every 10 x 17 ms needs 7.2 GB/s at margin 0.9 -> floor of half the link
     p = choose_pace(1_107_296_256, 10, 0.0171, 57.0)
-    assert p["d2h_gbs"] == 28.5 and p["d2h_quantum"] == D2H_QUANTUM
-    assert abs(p["need_gbs"] - 1_107_296_256 / (0.5 * 10 * 0.0171) / 1e9) < 1e-9
-    # a tighter interval raises the pace above the floor
-    p = choose_pace(1_107_296_256, 4, 0.0171, 57.0)
-    assert 28.5 < p["d2h_gbs"] < 57.0 and p["d2h_gbs"] == pytest.approx(p["need_gbs"])
-    # checkpointing every iteration needs more than the link: unpaced
-    assert choose_pace(1_107_296_256, 1, 0.0171, 57.0) == {"d2h_gbs": 0.0, "d2h_quantum": 0,
-                                                            "need_gbs": pytest.approx(129.5, rel=1e-3)}
-    # OPT-1.3B (15.8 GB every 10 x 43.8 ms): 72 GB/s at margin 0.5 exceeds the link -> unpaced by
-    # default; the optional stretch (max_margin 0.9, N >= 2) gives 40 GB/s; never with N = 1
-    p = choose_pace(15_789_098_512, 10, 0.0438, 57.0)
-    assert p["need_gbs"] == pytest.approx(72.1, rel=1e-2) and p["d2h_gbs"] == 0.0
-    p = choose_pace(15_789_098_512, 10, 0.0438, 57.0, max_margin=0.9)
-    assert p["d2h_gbs"] == pytest.approx(15_789_098_512 / (0.9 * 10 * 0.0438) / 1e9) and p["d2h_quantum"] == D2H_QUANTUM
-    assert choose_pace(15_789_098_512, 10, 0.0438, 57.0, max_margin=0.9, n_inflight=1)["d2h_gbs"] == 0.0
+    assert p["d2h_gbs"] == 28.5 and p["d2h_quantum"] == D2H_QUANTUM == 1 << 20
+    assert p["need_gbs"] == pytest.approx(1_107_296_256 / (0.9 * 10 * 0.0171) / 1e9)
+    # a tighter interval raises the pace above the floor, up to 0.7 of the link (eager)
+    p = choose_pace(1_107_296_256, 2, 0.0171, 57.0)
+    assert 28.5 < p["d2h_gbs"] <= 0.7 * 57.0 and p["d2h_gbs"] == pytest.approx(p["need_gbs"])
+    # beyond the cap: unpaced (every iteration needs more than the link)
+    p = choose_pace(1_107_296_256, 1, 0.0171, 57.0)
+    assert p["d2h_gbs"] == 0.0 and p["d2h_quantum"] == 0
+    # OPT-1.3B eager (15.8 GB every 10 x 44 ms): 39.9 GB/s at margin 0.9, under 0.7 x 57 = 39.9+
+    p = choose_pace(15_789_098_512, 10, 0.044, 57.0)
+    assert p["d2h_gbs"] == pytest.approx(15_789_098_512 / (0.9 * 10 * 0.044) / 1e9) and p["d2h_quantum"] == 1 << 20
+    # ... and 45 ms iterations with a 50 GB/s link would need more than 0.7 of it: unpaced
+    assert choose_pace(15_789_098_512, 10, 0.044, 50.0)["d2h_gbs"] == 0.0
+    # N = 1: a checkpoint must land within half its interval (nothing overlaps the next K1)
+    assert choose_pace(15_789_098_512, 10, 0.044, 57.0, n_inflight=1)["d2h_gbs"] == 0.0
     with pytest.raises(ValueError):
         choose_pace(1, 0, 1.0, 1.0)
-    # a CUDA-graph loop: land within 0.8 of the interval, 1 MiB copies (OPT-1.3B -> ~38 GB/s)
-    from paper_conf_asplos_strati0k25_b200.tuner import GRAPH_QUANTUM
+    # a CUDA-graph loop: margin and cap 0.85 (OPT-1.3B at 51.7 ms -> ~35.9 GB/s)
     p = choose_pace(15_789_098_512, 10, 0.0517, 56.7, graphs=True)
-    assert p["d2h_gbs"] == pytest.approx(15_789_098_512 / (0.8 * 10 * 0.0517) / 1e9) and p["d2h_quantum"] == GRAPH_QUANTUM
-    assert 28.35 < p["d2h_gbs"] < 56.7
+    assert p["d2h_gbs"] == pytest.approx(15_789_098_512 / (0.85 * 10 * 0.0517) / 1e9) and p["d2h_quantum"] == 1 << 20
+    assert 28.35 < p["d2h_gbs"] < 0.85 * 56.7
     assert choose_pace(15_789_098_512, 4, 0.0517, 56.7, graphs=True)["d2h_gbs"] == 0.0  # needs > the link
 
 
