@@ -91,7 +91,8 @@ def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, n_inflight:
     """D2H pace for training: {"d2h_gbs": G, "d2h_quantum": Q, "need_gbs": ...}; G = 0 = unpaced.
 
     The gentlest pace that lands one checkpoint within a margin of its interval f*t, never below
-    half the link, in 1 MiB copies; unpaced when that needs more than a cap of the link.  The
+    half the link nor above a cap of it, in 1 MiB copies; unpaced when even the capped pace
+    would not land the checkpoint within its interval.  The
     rule is the measured one (round 2, after the pacer was fixed to deliver its rate — the
     round-1 sweeps ran at ~1/3 of their nominal pace):
 
@@ -112,8 +113,8 @@ def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, n_inflight:
     if n_inflight < 2:
         margin = min(margin, 0.5)
     need = slice_bytes / (margin * f * t) / 1e9  # GB/s to land a checkpoint in margin * f * t
-    g = max(need, 0.5 * link_gbs)
-    if g > cap * link_gbs:
+    g = min(max(need, 0.5 * link_gbs), cap * link_gbs)
+    if slice_bytes / (g * 1e9) > f * t:  # even the capped pace outlasts the interval: unpaced
         return {"d2h_gbs": 0.0, "d2h_quantum": 0, "need_gbs": need}
     return {"d2h_gbs": g, "d2h_quantum": D2H_QUANTUM, "need_gbs": need}
 
