@@ -37,8 +37,9 @@ def test_choose_pace():
     assert p["d2h_gbs"] == pytest.approx(0.7 * 56.0) and p["d2h_quantum"] == 1 << 20
     # ... with a 50 GB/s link the capped 35 GB/s would need 451 ms > 440 ms: unpaced
     assert choose_pace(15_789_098_512, 10, 0.044, 50.0)["d2h_gbs"] == 0.0
-    # N = 1: a checkpoint must land within half its interval (nothing overlaps the next K1)
-    assert choose_pace(15_789_098_512, 10, 0.044, 57.0, n_inflight=1)["d2h_gbs"] == 0.0
+    # N = 1: the margin drops to half the interval (need 71.8 GB/s), so the pace is the cap
+    p = choose_pace(15_789_098_512, 10, 0.044, 57.0, n_inflight=1)
+    assert p["need_gbs"] == pytest.approx(15_789_098_512 / (0.5 * 10 * 0.044) / 1e9) and p["d2h_gbs"] == pytest.approx(39.9)
     with pytest.raises(ValueError):
         choose_pace(1, 0, 1.0, 1.0)
     # a CUDA-graph loop: margin and cap 0.85 (OPT-1.3B at 51.7 ms -> ~35.9 GB/s)
