@@ -105,6 +105,7 @@ struct Ckpt {
     std::atomic<uint32_t> remaining{0};
     cudaEvent_t ev_train = nullptr, ev_begin = nullptr, ev_packed = nullptr, ev_fin_k = nullptr, ev_final = nullptr;
     cudaEvent_t ev_landed = nullptr;  // copy stream, after the last chunk's D2H (timing)
+    std::atomic<bool> landed_recorded{false};  // (a failed checkpoint never records it)
     double t_call = 0, t_packed = 0, t_landed = 0, t_persisted = 0, t_committed = 0;
     float pack_ms = 0, fin_ms = 0, k1_busy_ms = 0, snap_ms = 0;
     // timing events around every K1 launch: the kernel's busy time, without the gaps in which
@@ -354,7 +355,8 @@ void finish_ckpt(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
     cudaEventElapsedTime(&ck->pack_ms, ck->ev_begin, ck->ev_packed);
     // K1 start -> last chunk in host memory, on the GPU's clock; Variant A's K1
     // stores into host memory itself
-    if (c->zerocopy() || c->n == 0 || cudaEventElapsedTime(&ck->snap_ms, ck->ev_begin, ck->ev_landed) != cudaSuccess)
+    if (c->zerocopy() || c->n == 0 || !ck->landed_recorded.load() ||
+        cudaEventElapsedTime(&ck->snap_ms, ck->ev_begin, ck->ev_landed) != cudaSuccess)
         ck->snap_ms = ck->pack_ms;
     ck->k1_busy_ms = 0;
     for (auto &p : ck->k1_ev) {
@@ -539,7 +541,10 @@ void orchestrate_loop(pcc_ctx *c) {
                     cudaEventRecord(qe, c->copy_stream);
                     queued.push_back(qe);
                 }
-                if (j + task.nchunks == c->n) cudaEventRecord(ck->ev_landed, c->copy_stream);  // before the task
+                if (j + task.nchunks == c->n) {  // before the task
+                    cudaEventRecord(ck->ev_landed, c->copy_stream);
+                    ck->landed_recorded = true;
+                }
                 task.ev = get_event(c);
                 task.pooled_ev = true;
                 cudaEventRecord(task.ev, c->copy_stream);
@@ -693,7 +698,10 @@ void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
                 cudaError_t e2 = cudaMemcpyAsync(task.dest, c->ring + r0 * c->cb(), (uint64_t)k * c->cb(),
                                                  cudaMemcpyDeviceToHost, c->copy_stream);
                 if (e2 != cudaSuccess) fail_ckpt(c, ck, cuda_error(e2, "D2H"));
-                if (j + k == c->n) cudaEventRecord(ck->ev_landed, c->copy_stream);
+                if (j + k == c->n) {
+                    cudaEventRecord(ck->ev_landed, c->copy_stream);
+                    ck->landed_recorded = true;
+                }
                 task.ev = get_event(c);
                 cudaEventRecord(task.ev, c->copy_stream);
                 c->tasks.push(task);
