@@ -140,16 +140,41 @@ constexpr uint32_t kNtBytes = (kG16 - 1) * kNtTab + (1u << kNtLastBits) * 128;
 constexpr uint32_t kRegTab = 32 * 128;               // bytes per full NF / NL table
 constexpr uint32_t kRegBytes = (kG32 - 1) * kRegTab + (1u << 2) * 128;
 
+// ------------------------------------------------ bank-rotated byte tables (the TMA kernels)
+// The TMA-staged K1/K2 (v7, kernels.cu k_snap_tma) compute the SAME lane registers as the
+// register-path kernel above, with byte-sliced tables that are conflict-free WITHOUT per-lane
+// replication.  Per round a lane's register becomes
+//     s' = raw32(span) ^ shift(s, 1024)          (the gap 992 + the span's own 32 bytes)
+// raw32(span) = XOR over the 32 byte positions k of T_k[byte k]; shift(s, 1024) = XOR over
+// the register's 4 bytes b of S_b[byte b].  Conflict-freedom comes from rotating the DATA, not
+// from replicating the tables: lane l holds its span rotated by l bytes (register i byte c =
+// span byte (4i + c + l) mod 32), so in the instruction for (i, c) lane l reads table
+// T_{(4i+c+l) mod 32}, and T_k lives in bank k: 32 lanes, 32 different banks.
+//   T2[v][P] (P = 0..63, 256-B rows) = T_{P mod 32}[v]: a lane's address is (v << 8) + 4l (one
+//            PRMT: byte c of the register next to 4l) + 4(4i + c) (the LDS immediate); the
+//            doubled row absorbs the wrap of 4i + c + l past 31.
+//   S4[v][4q + b'] (128-B rows) = S_{b'}[v] for each q = l >> 2: the register rotated by
+//            r = l & 3 bytes puts table S_{(c+r) & 3} at bank 4q + ((c + r) & 3).
+// 36 lookups per 32 B (51 above) in 96 KiB of tables (193 KiB above), which leaves shared
+// memory for a 128 KiB TMA staging ring.
+constexpr uint32_t kT2Bytes = 256 * 64 * 4;  // 64 KiB
+constexpr uint32_t kS4Bytes = 256 * 32 * 4;  // 32 KiB
+constexpr uint32_t kTmaTableBytes = kT2Bytes + kS4Bytes;
+
 // Table block.  K1/K2 load NT + NF (the first kK1TableBytes) into shared memory; NL is read by
 // the finalize kernel only.  Word index of entry (t, v, l): t*V*32 + v*32 + l inside each part.
+// The TMA kernels load T2 + S4 (kTmaTableBytes, contiguous).
 struct CrcTables {
     uint32_t NT[kNtBytes / 4];   // NT[t][v][l] = raw16(16-byte word whose bits [kNtBits*t, +kNtBits) are v)
     uint32_t NF[kRegBytes / 4];  // NF[g][v][l] = shift(v << 5g, kGap): the zeros before a lane's next span
     uint32_t NL[kRegBytes / 4];  // NL[g][v][l] = shift(v << 5g, kLaneRun*(31-l)): lane -> warp-region end
+    uint32_t T2[kT2Bytes / 4];   // T2[v*64 + P] = raw32(byte v at position P mod 32 of a 32-byte span)
+    uint32_t S4[kS4Bytes / 4];   // S4[v*32 + 4q + b] = shift(v << 8b, 1024)
 };
 constexpr uint32_t kK1TableBytes = kNtBytes + kRegBytes;
 static_assert(kK1TableBytes % 16 == 0, "TMA bulk copy size");
 static_assert(kK1TableBytes + 1024 <= 227 * 1024, "K1 shared memory");
+static_assert(kTmaTableBytes % 16 == 0 && (kNtBytes + 2 * kRegBytes) % 16 == 0, "TMA bulk copy size / alignment");
 
 // Constants that do not need a table.
 struct CrcConsts {

@@ -23,6 +23,8 @@
 //     GPU and k_chunk_crcs chunk shares -> chunk CRCs -> slice digest.
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <cstdlib>
+#include <cstring>
 #include <mutex>
 
 #include "kernels.hpp"
@@ -78,6 +80,18 @@ __global__ void k_build_tables(CrcTables *tb, CrcConsts *cs) {
         tb->NF[e] = vf[g][v];
         // NL: lane-specific shift kLaneRun*(31-l)
         tb->NL[e] = multmodp(x8n(x2n, kLaneRun * (31 - l)), (uint32_t)((uint64_t)v << (5 * g)));
+    }
+    // T2 / S4 (bank-rotated byte tables of the TMA kernels, crc32c.cuh)
+    for (uint32_t e = t; e < kT2Bytes / 4; e += blockDim.x) {
+        const uint32_t v = e >> 6, k = e & 31;  // position P = e & 63 holds T_{P mod 32}
+        uint32_t r = T0[v];
+        for (uint32_t z = 0; z < 31 - k; ++z) r = (r >> 8) ^ T0[r & 0xFF];
+        tb->T2[e] = r;
+    }
+    const uint32_t x1024 = x8n(x2n, 1024);
+    for (uint32_t e = t; e < kS4Bytes / 4; e += blockDim.x) {
+        const uint32_t v = e >> 5, b = e & 3;
+        tb->S4[e] = multmodp(x1024, v << (8 * b));
     }
     if (t < kX2n) cs->x2n[t] = x2n[t];
     if (t == 0) cs->x8n_stride = x8n(x2n, 32 * 16);
@@ -502,6 +516,483 @@ __global__ void __launch_bounds__(kThreadsOf<kPack>, 1) k_snapshot(const SnapPar
     }
 }
 
+// =============================================================== v7: TMA-staged K1 / K2
+// One persistent CTA per SM, warp-specialised around a ring of kStages 8 KiB staging slots in
+// shared memory (one slot = one work item = one 8 KiB tile of one chunk, as above):
+//   producer warp   K1: per item, one cp.async.bulk (global -> shared, mbarrier complete_tx) per
+//                   16-B aligned segment-row piece; ragged row tails, misaligned sources and
+//                   the zero pads are written by the warp's lanes; K2: one bulk copy of the
+//                   ring tile.  Row descriptors are fetched two batches of 32 items ahead.
+//   kCrcWarps       the CRC of the staged 8 KiB from shared memory with the bank-rotated byte
+//   consumer warps  tables (crc32c.cuh, 36 conflict-free LDS per 32 B): the SAME lane registers
+//                   as the register-path kernel, so the finalize kernels are shared.
+//   storer warp     K1: one cp.async.bulk (shared -> global, bulk_group) of the tile into the
+//                   chunk; K2: one per row piece (+ generic stores for tails / misaligned rows).
+//                   A slot is released once its store has finished READING shared memory
+//                   (wait_group.read, kStoreLag groups behind).
+// Per slot three mbarriers: full (producer arrive + tx bytes), computed (consumer), empty
+// (storer).  A ragged last tile (len < 8 KiB) sits right-aligned in its slot behind zeros:
+// leading zeros leave a zero-initialised CRC register unchanged, so the lanes' registers are
+// those of the tile relative to the chunk end, as the finalize kernel expects.
+constexpr int kStages = 16;                          // 16 x 8 KiB = 128 KiB of staging per SM
+#ifndef PCC_CRC_WARPS
+#define PCC_CRC_WARPS 8
+#endif
+constexpr int kCrcWarps = PCC_CRC_WARPS;
+#ifndef PCC_PRODUCERS
+#define PCC_PRODUCERS 2
+#endif
+#ifndef PCC_STORERS
+#define PCC_STORERS 2
+#endif
+constexpr int kProducers = PCC_PRODUCERS;            // producer warps: item k -> warp k % kProducers
+constexpr int kStorers = PCC_STORERS;                // storer warps: item k -> warp k % kStorers
+constexpr int kTmaThreads = (kCrcWarps + kProducers + kStorers) * 32;
+#ifndef PCC_STORE_LAG
+#define PCC_STORE_LAG 2
+#endif
+constexpr int kStoreLag = PCC_STORE_LAG;             // bulk-store groups still reading smem
+constexpr uint32_t kSlotsOff = kTmaTableBytes;
+constexpr uint32_t kBarsOff = kSlotsOff + kStages * kTile;
+constexpr uint32_t kTmaSmem = kBarsOff + (3 * kStages + 1) * 8;
+static_assert(kTmaSmem <= 227 * 1024, "TMA kernel shared memory");
+constexpr long long kWaitTrapCycles = 20000000000ll;  // ~10 s: a phase that never completes traps
+
+__device__ __forceinline__ uint32_t sm_addr(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ bool mbar_try(uint32_t bar, uint32_t parity) {
+    uint32_t done;
+    asm volatile(
+        "{\n.reg .pred p;\n"
+        "mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 p, [%1], %2;\n"
+        "selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done)
+        : "r"(bar), "r"(parity)
+        : "memory");
+    return done != 0;
+}
+// Bounded: a barrier phase that never completes (a bug) traps — the launch fails with an
+// error instead of hanging the GPU.
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+    if (mbar_try(bar, parity)) return;
+    const long long t0 = clock64();
+    while (!mbar_try(bar, parity))
+        if (clock64() - t0 > kWaitTrapCycles) __trap();
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t sdst, const void *src, uint32_t bytes, uint32_t bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(sdst),
+                 "l"(src), "r"(bytes), "r"(bar)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_s2g(void *dst, uint32_t ssrc, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(ssrc), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+// generic-proxy writes to shared memory -> visible to a later bulk copy that reads them
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
+    uint32_t r;
+    asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
+    return r;
+}
+__device__ __forceinline__ uint32_t ld_tab(const char *p) { return *reinterpret_cast<const uint32_t *>(p); }
+
+// Lane constants of the rotated-table CRC (crc32c.cuh): lane l = 4q + r.
+struct RotLane {
+    uint32_t O[8];   // byte offset of the word loaded into register i: 32l + 4((i + q) & 7)
+    uint32_t SB[4];  // S4 position of register byte c: 4(4q + ((c + r) & 3))
+    uint32_t L4, r8;
+    __device__ __forceinline__ explicit RotLane(uint32_t lane) {
+        const uint32_t q = lane >> 2, r = lane & 3;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) O[i] = 32 * lane + 4 * ((i + q) & 7);
+#pragma unroll
+        for (int c = 0; c < 4; ++c) SB[c] = 4 * (4 * q + ((c + r) & 3));
+        L4 = 4 * lane;
+        r8 = 8 * r;
+    }
+};
+
+// The lane registers of one staged 8 KiB tile (bit-identical to tile_fast's): per round,
+// s = raw32(span) ^ shift(s, 1024), span = the 32 bytes at 32l of the round.
+__device__ __forceinline__ uint32_t crc_tile_rot(const char *sl, const char *t2, const char *s4, const RotLane &L) {
+    uint32_t s = 0;
+#pragma unroll
+    for (int rho = 0; rho < kRounds; ++rho) {
+        uint32_t u[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) u[i] = *reinterpret_cast<const uint32_t *>(sl + rho * kRound + L.O[i]);
+        uint32_t acc = 0;
+        if (rho > 0) {  // shift(s, 1024): the register rotated right by r bytes, byte c -> S_{(c+r)&3}
+            const uint32_t x = __funnelshift_r(s, s, L.r8);
+            acc = ld_tab(s4 + grp_off<0x7F80u>(x << 7, L.SB[0])) ^ ld_tab(s4 + grp_off<0x7F80u>(x >> 1, L.SB[1])) ^
+                  ld_tab(s4 + grp_off<0x7F80u>(x >> 9, L.SB[2])) ^ ld_tab(s4 + grp_off<0x7F80u>(x >> 17, L.SB[3]));
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            // register i byte c = span byte (4i + c + l) mod 32; T2 row position 4i + c + l
+            const uint32_t w = funnel_r(u[i], u[(i + 1) & 7], L.r8);
+            const char *ti = t2 + 16 * i;
+            acc ^= ld_tab(ti + 0 + prmt(w, L.L4, 0x7604u)) ^ ld_tab(ti + 4 + prmt(w, L.L4, 0x7614u)) ^
+                   ld_tab(ti + 8 + prmt(w, L.L4, 0x7624u)) ^ ld_tab(ti + 12 + prmt(w, L.L4, 0x7634u));
+        }
+        s = acc;
+    }
+    return s;
+}
+
+__device__ __forceinline__ void zero_smem(char *sl, uint32_t a, uint32_t b, uint32_t lane) {  // [a, b), 16-B aligned
+    for (uint32_t o = a + 16 * lane; o < b; o += 512) *reinterpret_cast<uint4 *>(sl + o) = make_uint4(0, 0, 0, 0);
+}
+
+// Item descriptors fetched ahead in batches of 32 (lane i <-> the batch's i-th item of this
+// CTA): the tile's row range and its first row.  Two batches ahead for the row range, one for
+// the first row (which depends on it), so neither load latency sits on the producer's path.
+struct DescBatch {
+    uint2 tr;    // x = first row index, y = rows overlapping the tile
+    SegRow r0;   // first row (valid when tr.y > 0)
+};
+__device__ __forceinline__ uint2 desc_tr(const SnapParams &P, uint32_t item, uint32_t n_items) {
+    return item_rows(P, item, n_items);
+}
+
+// Geometry of an item (chunk-local index jl, tile t): chunk, tile start, bytes, lead of its slot
+struct ItemGeo {
+    uint32_t j, len, lead;
+    uint64_t tile0;
+    __device__ __forceinline__ ItemGeo(const SnapParams &P, uint32_t jl, uint32_t t) {
+        j = P.first + jl;
+        tile0 = (uint64_t)t * kTile;
+        const uint64_t rem = P.chunk_bytes - tile0;
+        len = rem < kTile ? (uint32_t)rem : kTile;
+        lead = kTile - len;
+    }
+};
+
+// The items of one role warp: k = r, r + nr, ... of this CTA, item = blockIdx.x + k * G, with
+// (jl, t) = divmod(item, tpc) kept incrementally (one division at the start, none per item).
+struct RoleIter {
+    uint32_t k, item, jl, t;
+    uint32_t nr, step, sjl, st, tpc;
+    __device__ __forceinline__ RoleIter(const SnapParams &P, uint32_t r, uint32_t nr_) {
+        nr = nr_;
+        tpc = P.tpc;
+        k = r;
+        item = blockIdx.x + r * gridDim.x;
+        jl = item / tpc;
+        t = item - jl * tpc;
+        step = nr * gridDim.x;
+        sjl = step / tpc;
+        st = step - sjl * tpc;
+    }
+    __device__ __forceinline__ void next() {
+        k += nr;
+        item += step;
+        jl += sjl;
+        t += st;
+        if (t >= tpc) {
+            t -= tpc;
+            ++jl;
+        }
+    }
+};
+
+// One row piece of a tile: chunk range [lo, hi) of the row, its address at lo.
+struct Piece {
+    uint32_t s_off, n;  // slot offset and bytes
+    uint64_t addr;      // tensor address of the piece's first byte
+    bool ok;            // non-empty
+};
+__device__ __forceinline__ Piece piece_of(const SegRow &r, const ItemGeo &g) {
+    Piece p;
+    const uint64_t lo = r.dst_off > g.tile0 ? r.dst_off : g.tile0;
+    const uint64_t re = (uint64_t)r.dst_off + r.len, te = g.tile0 + g.len;
+    const uint64_t hi = re < te ? re : te;
+    p.ok = hi > lo;
+    p.n = p.ok ? (uint32_t)(hi - lo) : 0;
+    p.s_off = g.lead + (uint32_t)(lo - g.tile0);
+    p.addr = r.ptr + (lo - r.dst_off);
+    return p;
+}
+// slot offset where row i's piece starts (tile end when there is no such row)
+__device__ __forceinline__ uint32_t piece_start(const SegRow &r, const ItemGeo &g) {
+    const uint64_t lo = r.dst_off > g.tile0 ? r.dst_off : g.tile0;
+    return g.lead + (uint32_t)(lo - g.tile0);
+}
+
+// K1 producer: fill the slot with the tile's image bytes, ending with the full barrier's
+// producer arrival.  Generic writes first (ragged row tails, pads, misaligned rows), then —
+// only if there were any inside the tile — ONE proxy fence, then the bulk copies: the fence is
+// a MEMBAR that waits for this thread's outstanding bulk copies too, so it must stay off the
+// common path (a tile inside one aligned tensor: one bulk copy, no generic write, no fence).
+__device__ __forceinline__ void fill_pack(const SnapParams &P, const ItemGeo &g, uint2 tr, const SegRow &r0,
+                                          char *sl, uint32_t full, uint32_t lane) {
+    const uint32_t ssl = sm_addr(sl);
+    const uint32_t nrows = tr.y;
+    const SegRow *rows = P.rows + tr.x;
+    if (nrows == 1) {  // the common case: one aligned row covers the tile -> one bulk copy
+        const Piece p = piece_of(r0, g);
+        if (p.s_off == g.lead && p.n == g.len && (p.addr & 15) == 0) {
+            zero_smem(sl, 0, g.lead, lane);  // ragged tile: zeros the CRC reads, the store does not
+            __syncwarp();
+            if (lane == 0) {
+                mbar_expect_tx(full, p.n);
+                bulk_g2s(ssl + p.s_off, reinterpret_cast<const void *>(p.addr), p.n, full);
+                mbar_arrive(full);
+            }
+            return;
+        }
+    }
+    // pass 1: bytes the bulk copies will deliver (16-B aligned source, whole 16-B words)
+    uint32_t bulk = 0;
+    for (uint32_t i = lane; i < nrows; i += 32) {
+        const SegRow r = i == 0 ? r0 : ld_row(rows + i);
+        const Piece p = piece_of(r, g);
+        if (p.ok && (p.addr & 15) == 0) bulk += p.n & ~15u;
+    }
+    bulk = __reduce_add_sync(0xFFFFFFFFu, bulk);
+    if (lane == 0 && bulk) mbar_expect_tx(full, bulk);
+    // pass 2: generic writes
+    uint32_t first_start = g.lead + g.len, last_end = g.lead;  // leading / trailing pads
+    if (nrows) {
+        first_start = piece_start(r0, g);
+        const SegRow rl = nrows == 1 ? r0 : ld_row(rows + nrows - 1);
+        const Piece pl = piece_of(rl, g);
+        last_end = pl.s_off + ((pl.n + 15) & ~15u);
+    }
+    bool gen = first_start > g.lead || last_end < kTile;
+    for (uint32_t i0 = 0; i0 < nrows; i0 += 32) {
+        const uint32_t i = i0 + lane;
+        bool mis = false;
+        if (i < nrows) {
+            const SegRow r = i == 0 ? r0 : ld_row(rows + i);
+            const Piece p = piece_of(r, g);
+            if (p.ok) {
+                if ((p.addr & 15) == 0) {
+                    const uint32_t b = p.n & ~15u;
+                    if (p.n > b) {
+                        *reinterpret_cast<uint4 *>(sl + p.s_off + b) = load_bytes(p.addr + b, p.n - b);
+                        gen = true;
+                    }
+                } else {
+                    mis = gen = true;
+                }
+                if (i + 1 < nrows) {  // the pad up to the next row's piece
+                    const uint32_t a = p.s_off + ((p.n + 15) & ~15u);
+                    const uint32_t e = piece_start(ld_row(rows + i + 1), g);
+                    for (uint32_t o = a; o < e; o += 16) *reinterpret_cast<uint4 *>(sl + o) = make_uint4(0, 0, 0, 0);
+                    gen |= e > a;
+                }
+            }
+        }
+        // misaligned sources: the whole warp, 16-B words gathered byte- or word-wise
+        uint32_t m = __ballot_sync(0xFFFFFFFFu, mis);
+        while (m) {
+            const uint32_t src_lane = __ffs(m) - 1;
+            m &= m - 1;
+            const Piece p = piece_of(ld_row(rows + i0 + src_lane), g);
+            for (uint32_t w = 16 * lane; w < p.n; w += 512) {
+                const uint32_t k = p.n - w < 16 ? p.n - w : 16;
+                *reinterpret_cast<uint4 *>(sl + p.s_off + w) = load_bytes(p.addr + w, k);
+            }
+        }
+    }
+    zero_smem(sl, 0, first_start, lane);
+    zero_smem(sl, last_end, kTile, lane);
+    if (__any_sync(0xFFFFFFFFu, gen)) fence_proxy_async();  // generic writes -> the storer's bulk store
+    // pass 3: the bulk copies
+    for (uint32_t i = lane; i < nrows; i += 32) {
+        const SegRow r = i == 0 ? r0 : ld_row(rows + i);
+        const Piece p = piece_of(r, g);
+        const uint32_t b = p.n & ~15u;
+        if (p.ok && (p.addr & 15) == 0 && b) bulk_g2s(ssl + p.s_off, reinterpret_cast<const void *>(p.addr), b, full);
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(full);
+}
+
+// K2 producer: the ring tile in one bulk copy (generic loads if the ring is not 16-B aligned)
+__device__ __forceinline__ void fill_unpack(const SnapParams &P, const ItemGeo &g, char *sl, uint32_t full,
+                                            uint32_t lane) {
+    const char *src = P.ring_base + ((P.ring_head + g.j) % P.ring_slots) * P.chunk_bytes + g.tile0;
+    if ((reinterpret_cast<uintptr_t>(src) & 15) == 0) {
+        if (lane == 0) {
+            mbar_expect_tx(full, g.len);
+            bulk_g2s(sm_addr(sl) + g.lead, src, g.len, full);
+        }
+    } else {
+        for (uint32_t w = 16 * lane; w < g.len; w += 512)
+            *reinterpret_cast<uint4 *>(sl + g.lead + w) = load_bytes(reinterpret_cast<uint64_t>(src) + w, 16);
+    }
+    zero_smem(sl, 0, g.lead, lane);
+    __syncwarp();
+    if (lane == 0) mbar_arrive(full);
+}
+
+// K2 storer: scatter the verified tile's row pieces to the tensors.  Every lane commits one
+// bulk group per item (possibly empty) so that the lanes' group counts stay in step.
+__device__ __forceinline__ void drain_unpack(const SnapParams &P, const ItemGeo &g, uint2 tr, const SegRow &r0,
+                                             const char *sl, uint32_t lane) {
+    const uint32_t ssl = sm_addr(sl);
+    const uint32_t nrows = tr.y;
+    const SegRow *rows = P.rows + tr.x;
+    for (uint32_t i0 = 0; i0 < nrows; i0 += 32) {
+        const uint32_t i = i0 + lane;
+        bool mis = false;
+        if (i < nrows) {
+            const SegRow r = i == 0 ? r0 : ld_row(rows + i);
+            const Piece p = piece_of(r, g);
+            if (p.ok) {
+                if ((p.addr & 15) == 0) {
+                    const uint32_t b = p.n & ~15u;
+                    if (b) bulk_s2g(reinterpret_cast<void *>(p.addr), ssl + p.s_off, b);
+                    if (p.n > b)
+                        store_bytes(p.addr + b, p.n - b, *reinterpret_cast<const uint4 *>(sl + p.s_off + b));
+                } else {
+                    mis = true;
+                }
+            }
+        }
+        uint32_t m = __ballot_sync(0xFFFFFFFFu, mis);
+        while (m) {
+            const uint32_t src_lane = __ffs(m) - 1;
+            m &= m - 1;
+            const Piece p = piece_of(ld_row(rows + i0 + src_lane), g);
+            for (uint32_t w = 16 * lane; w < p.n; w += 512) {
+                const uint32_t k = p.n - w < 16 ? p.n - w : 16;
+                store_bytes(p.addr + w, k, *reinterpret_cast<const uint4 *>(sl + p.s_off + w));
+            }
+        }
+    }
+    bulk_commit();
+}
+
+template <bool kPack>
+__global__ void __launch_bounds__(kTmaThreads, 1) k_snap_tma(const SnapParams P) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    const char *t2 = reinterpret_cast<const char *>(smem);
+    const char *s4 = t2 + kT2Bytes;
+    char *slots = reinterpret_cast<char *>(smem) + kSlotsOff;
+    const uint32_t bars = sm_addr(smem + kBarsOff);  // full[kStages], computed[kStages], empty[kStages], tables
+    auto full = [&](uint32_t s) { return bars + 8 * s; };
+    auto computed = [&](uint32_t s) { return bars + 8 * (kStages + s); };
+    auto empty = [&](uint32_t s) { return bars + 8 * (2 * kStages + s); };
+    const uint32_t tbar = bars + 8 * (3 * kStages);
+    const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t n_items = P.count * P.tpc;
+    const uint32_t G = gridDim.x;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < kStages; ++s) {
+            mbar_init(full(s), 1);
+            mbar_init(computed(s), 1);
+            mbar_init(empty(s), 1);
+        }
+        mbar_init(tbar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        mbar_expect_tx(tbar, kTmaTableBytes);
+        bulk_g2s(sm_addr(smem), &P.tables->T2[0], kTmaTableBytes, tbar);
+        mbar_arrive(tbar);
+    }
+    __syncthreads();  // barriers initialised
+
+    const uint64_t crc_base = (uint64_t)P.first * P.tpc;  // tile_crc item index = first*tpc + item
+    if (warp < (uint32_t)kCrcWarps) {  // ---------------------------------------- consumers
+        const RotLane L(lane);
+        mbar_wait(tbar, 0);
+        uint32_t k = warp;
+        for (uint32_t item = blockIdx.x + warp * G; item < n_items; item += kCrcWarps * G, k += kCrcWarps) {
+            const uint32_t s = k % kStages, use = k / kStages;
+            mbar_wait(full(s), use & 1);
+#ifdef PCC_EXP_NOCRC  // timing experiment only: the staging pipeline without the CRC (wrong CRCs)
+            const uint32_t v = *reinterpret_cast<const uint32_t *>(slots + s * kTile + 4 * lane);
+#else
+            const uint32_t v = crc_tile_rot(slots + s * kTile, t2, s4, L);
+#endif
+            __syncwarp();
+            if (lane == 0) mbar_arrive(computed(s));
+            P.tile_crc[(crc_base + item) * kLaneOut + lane] = v;
+        }
+        return;
+    }
+    const bool producer = warp < (uint32_t)(kCrcWarps + kProducers);
+    const uint32_t r = producer ? warp - kCrcWarps : warp - kCrcWarps - kProducers;  // rank within the role
+    const uint32_t nr = producer ? kProducers : kStorers;
+    // row descriptors in batches of 32 of this warp's items (K1 producers, K2 storers)
+    const bool need_desc = producer == kPack;
+    auto batch_item = [&](uint32_t m) { return blockIdx.x + (r + nr * m) * G; };
+    DescBatch cur{}, nxt{};
+    uint2 tr_nn = make_uint2(0, 0);
+    if (need_desc) {
+        cur.tr = desc_tr(P, batch_item(lane), n_items);
+        if (cur.tr.y) cur.r0 = ld_row(P.rows + cur.tr.x);
+        nxt.tr = desc_tr(P, batch_item(32 + lane), n_items);
+    }
+    RoleIter it(P, r, nr);
+    uint32_t m = 0;  // this warp's item count
+    for (uint32_t b = 0; it.item < n_items; ++b) {
+        if (need_desc) {  // first rows of the next batch, row ranges of the one after
+            if (nxt.tr.y) nxt.r0 = ld_row(P.rows + nxt.tr.x);
+            tr_nn = desc_tr(P, batch_item(32 * (b + 2) + lane), n_items);
+        }
+        for (uint32_t ii = 0; ii < 32 && it.item < n_items; ++ii, ++m, it.next()) {
+            const uint32_t k = it.k, s = k % kStages, use = k / kStages;
+            const ItemGeo g(P, it.jl, it.t);
+            uint2 tr = make_uint2(0, 0);
+            SegRow r0{};
+            if (need_desc) {
+                tr.x = __shfl_sync(0xFFFFFFFFu, cur.tr.x, ii);
+                tr.y = __shfl_sync(0xFFFFFFFFu, cur.tr.y, ii);
+                r0.ptr = __shfl_sync(0xFFFFFFFFu, cur.r0.ptr, ii);
+                r0.dst_off = __shfl_sync(0xFFFFFFFFu, cur.r0.dst_off, ii);
+                r0.len = __shfl_sync(0xFFFFFFFFu, cur.r0.len, ii);
+            }
+            if (producer) {  // ------------------------------------------------ producers
+                if (use) mbar_wait(empty(s), (use - 1) & 1);
+                if (kPack)
+                    fill_pack(P, g, tr, r0, slots + s * kTile, full(s), lane);
+                else
+                    fill_unpack(P, g, slots + s * kTile, full(s), lane);
+            } else {  // ------------------------------------------------------------- storers
+                mbar_wait(computed(s), use & 1);
+                mbar_wait(full(s), use & 1);  // (complete already) the bulk load's bytes, observed directly
+                if (kPack) {
+                    if (lane == 0) {
+                        char *dst = P.ring_base + ((P.ring_head + g.j) % P.ring_slots) * P.chunk_bytes + g.tile0;
+                        bulk_s2g(dst, sm_addr(slots + s * kTile) + g.lead, g.len);
+                        bulk_commit();
+                    }
+                } else {
+                    drain_unpack(P, g, tr, r0, slots + s * kTile, lane);
+                }
+                if (m >= (uint32_t)kStoreLag) {  // this warp's store of kStoreLag items ago has read its slot
+                    if (kPack ? lane == 0 : true) bulk_wait_read<kStoreLag>();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(empty((k - kStoreLag * nr) % kStages));
+                }
+            }
+        }
+        cur = nxt;
+        nxt.tr = tr_nn;
+    }
+    if (!producer) bulk_wait_all();  // smem stays allocated until every bulk store has completed
+}
+
 // lanes -> sub-tiles -> chunk CRC (+ verify) -> slice digest, in two kernels so that the whole
 // GPU shares the work (one CTA per chunk left most SMs idle: 33 us for the 66 chunks of C2).
 //
@@ -663,25 +1154,39 @@ void free_geometry(DevGeometry *g) {
     g->tile_shift = g->chunk_shift = g->ff = nullptr;
 }
 
+// PCC_KIMPL=v6 selects the register-path K1/K2 (A/B builds on one box); default: the TMA kernels
+static bool use_v6() {
+    static const bool v6 = [] {
+        const char *e = getenv("PCC_KIMPL");
+        return e && strcmp(e, "v6") == 0;
+    }();
+    return v6;
+}
+
 template <bool kPack>
 static int resident_ctas(int device) {
     static int cached[64] = {};
     if (device < 0 || device >= 64) return 1;
     if (!cached[device]) {
         int per_sm = 0, sms = 0;
-        cudaFuncSetAttribute(k_snapshot<kPack>, cudaFuncAttributeMaxDynamicSharedMemorySize, kK1TableBytes);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snapshot<kPack>, kThreadsOf<kPack>, kK1TableBytes);
+        if (use_v6()) {
+            cudaFuncSetAttribute(k_snapshot<kPack>, cudaFuncAttributeMaxDynamicSharedMemorySize, kK1TableBytes);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snapshot<kPack>, kThreadsOf<kPack>, kK1TableBytes);
+        } else {
+            cudaFuncSetAttribute(k_snap_tma<kPack>, cudaFuncAttributeMaxDynamicSharedMemorySize, kTmaSmem);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_snap_tma<kPack>, kTmaThreads, kTmaSmem);
+        }
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
         cached[device] = (per_sm > 0 ? per_sm : 1) * (sms > 0 ? sms : 1);
     }
     return cached[device];
 }
 
-// n_items = 8 KiB tiles (one warp each)
+// n_items = 8 KiB tiles (one warp each in v6; one staging slot each in the TMA kernels)
 int snapshot_grid(int device, uint32_t n_items, uint32_t cap, bool pack) {
     int g = pack ? resident_ctas<true>(device) : resident_ctas<false>(device);
     if (cap && (int)cap < g) g = (int)cap;
-    const uint32_t w = pack ? kWarpsOf<true> : kWarpsOf<false>;
+    const uint32_t w = use_v6() ? (pack ? kWarpsOf<true> : kWarpsOf<false>) : 1;
     const uint32_t need = (n_items + w - 1) / w;
     if ((uint32_t)g > need) g = (int)need;
     return g < 1 ? 1 : g;
@@ -689,13 +1194,19 @@ int snapshot_grid(int device, uint32_t n_items, uint32_t cap, bool pack) {
 
 cudaError_t launch_pack(const SnapParams &p, int grid, cudaStream_t s) {
     if (p.count == 0) return cudaSuccess;
-    k_snapshot<true><<<grid, kThreadsOf<true>, kK1TableBytes, s>>>(p);
+    if (use_v6())
+        k_snapshot<true><<<grid, kThreadsOf<true>, kK1TableBytes, s>>>(p);
+    else
+        k_snap_tma<true><<<grid, kTmaThreads, kTmaSmem, s>>>(p);
     return cudaGetLastError();
 }
 
 cudaError_t launch_unpack(const SnapParams &p, int grid, cudaStream_t s) {
     if (p.count == 0) return cudaSuccess;
-    k_snapshot<false><<<grid, kThreadsOf<false>, kK1TableBytes, s>>>(p);
+    if (use_v6())
+        k_snapshot<false><<<grid, kThreadsOf<false>, kK1TableBytes, s>>>(p);
+    else
+        k_snap_tma<false><<<grid, kTmaThreads, kTmaSmem, s>>>(p);
     return cudaGetLastError();
 }
 
@@ -709,8 +1220,13 @@ cudaError_t warm_kernels(int device, const CrcTables *tables) {
     SnapParams P{};  // count = 0: the table load, then no work item
     P.tables = tables;
     P.tpc = 1;
-    k_snapshot<true><<<1, kThreadsOf<true>, kK1TableBytes>>>(P);
-    k_snapshot<false><<<1, kThreadsOf<false>, kK1TableBytes>>>(P);
+    if (use_v6()) {
+        k_snapshot<true><<<1, kThreadsOf<true>, kK1TableBytes>>>(P);
+        k_snapshot<false><<<1, kThreadsOf<false>, kK1TableBytes>>>(P);
+    } else {
+        k_snap_tma<true><<<1, kTmaThreads, kTmaSmem>>>(P);
+        k_snap_tma<false><<<1, kTmaThreads, kTmaSmem>>>(P);
+    }
     FinalizeParams F{};  // n = 0: no chunk
     F.tables = tables;
     F.tpc = 1;

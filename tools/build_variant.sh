@@ -11,4 +11,4 @@ for f in runtime commit kapi host_api; do
       -fvisibility=hidden "$@" -c paper_conf_asplos_strati0k25_b200/csrc/$f.cpp -o build/$name/$f.o
 done
 g++ -shared -o build/$name/libpccheck.so build/$name/*.o -L/usr/local/cuda/lib64 -lcudart_static -ldl -lpthread -lrt -Wl,--exclude-libs,ALL
-grep -A1 "k_snapshotILb1" build/$name/ptxas.log | grep -oE "Used [0-9]+ registers|[0-9]+ bytes spill stores" | tr '\n' ' '; echo " <- $name $*"
+grep -A1 "k_snap_tmaILb1" build/$name/ptxas.log | grep -oE "Used [0-9]+ registers|[0-9]+ bytes spill stores" | tr '\n' ' '; echo " <- $name $*"
