@@ -616,10 +616,10 @@ def main():
             "snapshot_idle": {"ms": idle_ms, "gbs": rank_state_bytes / (idle_ms * 1e-3) / 1e9,
                               "def": "K1 start -> last chunk landed in host memory, CUDA events, one checkpoint "
                                      "in flight, median of the warm-up checkpoints after the first"},
-            "roofline": {"bound": "hbm", "kernel": "k_snapshot<pack> (K1)", "achieved": k1_achieved,
+            "roofline": {"bound": "hbm", "kernel": "k_snap_tma<pack> (K1 v7)" if os.environ.get("PCC_KIMPL") != "v6" else "k_snapshot<pack> (K1 v6)", "achieved": k1_achieved,
                          "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": k1_achieved / peaks["hbm_gbs"],
                          # ncu's DRAM bytes of one W = 1 launch (profiles/k1_traffic.json)
-                         "traffic": load_traffic(f"{args.config}_k1") if world == 1 and not emu else None,
+                         "traffic": load_traffic(f"{args.config}_k1" + ("_v6" if os.environ.get("PCC_KIMPL") == "v6" else "")) if world == 1 and not emu else None,
                          "algorithmic_bytes_per_checkpoint": k1_bytes, "k1_ms_per_checkpoint": k1_ms,
                          "k1_launches_per_checkpoint": (launches - 2 * args.steps) / args.steps,  # minus the 2 finalize kernels
                          "pack_span_ms": pack_ms,

@@ -8,7 +8,13 @@
 // load of L287 §4.2 with verification (R13).  No floating point is involved: bytes are
 // moved verbatim, so NaN payloads / denormals survive (R1).
 //
-// Execution model:
+// Two implementations of K1/K2 with bit-identical outputs:
+//   * v7 k_snap_tma (default): a TMA-staged ring of 8 KiB slots per SM, warp-specialised
+//     (bulk-copy producers, CRC warps with bank-rotated byte tables, bulk-copy storers) — see
+//     the block comment above k_snap_tma;
+//   * v6 k_snapshot (PCC_KIMPL=v6, same-box A/B): the register path described next.
+//
+// v6 execution model:
 //   * one CTA of 32 warps per SM (the tables fill its shared memory); the work item is an
 //     8 KiB tile of one chunk, owned by one warp; warps stride over the items independently
 //     (no block barrier after the TMA table load); grid = SMs (or the pack_ctas cap);

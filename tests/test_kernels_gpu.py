@@ -160,3 +160,106 @@ def test_nccl_transport_selftest(pcc):
     vals = [30, -1, 2**40 + 5, 0, 7]
     mn, mx, ok = pcc.nccl_selftest(vals)
     assert mn == vals and mx == vals and ok
+
+
+def _unpack_gpu(pcc, outs, img, crc, align, cb):
+    c = crc.numel()
+    bad = torch.zeros(c, dtype=torch.int32, device="cuda")
+    nbad = torch.zeros(1, dtype=torch.int32, device="cuda")
+    dig = torch.zeros(1, dtype=torch.int32, device="cuda")
+    pcc.k_unpack(outs, img.data_ptr(), crc.data_ptr(), bad.data_ptr(), nbad.data_ptr(), dig.data_ptr(), align, cb)
+    torch.cuda.synchronize()
+    return int(nbad.item()), int(dig.cpu().numpy().view(np.uint32)[0])
+
+
+@pytest.mark.parametrize("cb", [64 << 10, 32768 + 16, 3 * 32768 - 16, 48])
+def test_unpack_into_misaligned_views_ragged_chunks(pcc, cb):
+    """K2's scatter: destinations at every byte alignment 0..15 with ragged lengths, chunk sizes
+    whose last 8 KiB tile is ragged; every byte outside the views must stay untouched."""
+    rng = np.random.default_rng(21)
+    src_base = torch.randint(0, 256, (1 << 20,), dtype=torch.uint8, device="cuda")
+    dst_base = torch.full((1 << 20,), 0x3C, dtype=torch.uint8, device="cuda")
+    srcs, dsts, pos, spans = [], [], 0, []
+    for k in range(40):
+        a = int(rng.integers(0, 16))
+        n = int(rng.integers(0, 20000))
+        start = ((pos + 4095) // 4096) * 4096 + a
+        srcs.append(src_base[start:start + n])
+        dsts.append(dst_base[start:start + n])
+        spans.append((start, n))
+        pos = start + n
+    off, end, c = pcc.k_layout(srcs, 256, cb)
+    img = torch.empty(max(1, c * cb), dtype=torch.uint8, device="cuda")
+    crc = torch.zeros(max(1, c), dtype=torch.int32, device="cuda")
+    dig = torch.zeros(1, dtype=torch.int32, device="cuda")
+    pcc.k_pack(srcs, img.data_ptr(), crc.data_ptr(), dig.data_ptr(), 256, cb)
+    o_img, o_crcs, o_dig = _oracle_side(srcs, 256, cb)
+    assert np.array_equal(img[:c * cb].cpu().numpy(), o_img)
+    nbad, dig2 = _unpack_gpu(pcc, dsts, img, crc[:c], 256, cb)
+    assert nbad == 0 and dig2 == o_dig
+    expect = np.full(1 << 20, 0x3C, dtype=np.uint8)
+    sb = src_base.cpu().numpy()
+    for start, n in spans:
+        expect[start:start + n] = sb[start:start + n]
+    got = dst_base.cpu().numpy()
+    assert np.array_equal(got, expect), f"{np.count_nonzero(got != expect)} bytes differ"
+
+
+def test_many_rows_per_tile_align16(pcc):
+    """align 16 and tiny tensors: up to hundreds of segment rows inside one 8 KiB tile (the
+    producer / storer loop over rows in groups of 32), tiles that are all padding, ragged rows."""
+    rng = np.random.default_rng(9)
+    sizes = [int(x) for x in rng.integers(0, 90, 3000)]
+    sizes[100:140] = [0] * 40
+    ts = [torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda") for n in sizes]
+    ts.append(torch.empty(0, dtype=torch.uint8, device="cuda"))
+    for cb in (64 << 10, 8192 + 16 * 7):
+        img, crcs, dig = _pack_gpu(pcc, ts, 16, cb)
+        o_img, o_crcs, o_dig = _oracle_side(ts, 16, cb)
+        assert np.array_equal(img, o_img) and crcs == o_crcs and dig == o_dig
+        outs = [torch.zeros_like(t) for t in ts]
+        off, end, c = pcc.k_layout(ts, 16, cb)
+        g_img = torch.from_numpy(o_img).cuda()
+        g_crc = torch.tensor(np.array(o_crcs, dtype=np.uint32).view(np.int32), device="cuda")
+        nbad, dig2 = _unpack_gpu(pcc, outs, g_img, g_crc, 16, cb)
+        assert nbad == 0 and dig2 == o_dig
+        assert all(np.array_equal(host_bytes(a), host_bytes(b)) for a, b in zip(ts, outs))
+
+
+def test_padding_only_tiles(pcc):
+    """A 4096-B alignment leaves whole 8 KiB tiles without any row (all zeros in the image)."""
+    ts = [torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda") for n in (5, 70000, 1, 24577)]
+    img, crcs, dig = _pack_gpu(pcc, ts, 65536, 1 << 20)
+    o_img, o_crcs, o_dig = _oracle_side(ts, 65536, 1 << 20)
+    assert np.array_equal(img, o_img) and crcs == o_crcs and dig == o_dig
+
+
+def test_register_path_kernels_v6_parity():
+    """PCC_KIMPL=v6 (the register-path K1/K2 kept for same-box A/B) in its own process: C1 full
+    image + CRC table + digest vs the oracle, and a K2 round trip."""
+    import subprocess
+    import sys
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    code = (
+        "import sys, numpy as np, torch; sys.path.insert(0, %r); sys.path.insert(0, %r)\n"
+        "import oracle, paper_conf_asplos_strati0k25_b200 as pcc\n"
+        "from synth import config_tensors, make_state, host_bytes\n"
+        "ts = make_state(config_tensors('c1'), 'cuda', seed=3, it=1); cb = 32768 + 16\n"
+        "off, end, c = pcc.k_layout(ts, 256, cb)\n"
+        "img = torch.empty(c * cb, dtype=torch.uint8, device='cuda'); crc = torch.zeros(c, dtype=torch.int32, device='cuda')\n"
+        "dig = torch.zeros(1, dtype=torch.int32, device='cuda')\n"
+        "pcc.k_pack(ts, img.data_ptr(), crc.data_ptr(), dig.data_ptr(), 256, cb); torch.cuda.synchronize()\n"
+        "hb = [host_bytes(t) for t in ts]; o = oracle.pack(hb, 256, cb)\n"
+        "assert np.array_equal(img.cpu().numpy(), o)\n"
+        "assert crc.cpu().numpy().view(np.uint32).tolist() == [int(x) for x in oracle.chunk_crcs(o, cb)]\n"
+        "assert int(dig.cpu().numpy().view(np.uint32)[0]) == oracle.crc32c(o)\n"
+        "outs = [torch.zeros_like(t) for t in ts]; bad = torch.zeros(c, dtype=torch.int32, device='cuda')\n"
+        "aux = torch.zeros(2, dtype=torch.int32, device='cuda')\n"
+        "pcc.k_unpack(outs, img.data_ptr(), crc.data_ptr(), bad.data_ptr(), aux.data_ptr(), aux[1:].data_ptr(), 256, cb)\n"
+        "torch.cuda.synchronize(); assert int(aux[0].item()) == 0\n"
+        "assert all(np.array_equal(host_bytes(a), b) for a, b in zip(outs, hb))\n"
+        "print('v6 ok')\n") % (ROOT, os.path.join(ROOT, "tests"))
+    env = dict(os.environ, PCC_KIMPL="v6")
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0 and "v6 ok" in r.stdout, r.stdout + r.stderr
