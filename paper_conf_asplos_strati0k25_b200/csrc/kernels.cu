@@ -563,6 +563,18 @@ constexpr uint32_t kBarsOff = kSlotsOff + kStages * kTile;
 constexpr uint32_t kTmaSmem = kBarsOff + (3 * kStages + 1) * 8;
 static_assert(kTmaSmem <= 227 * 1024, "TMA kernel shared memory");
 constexpr long long kWaitTrapCycles = 20000000000ll;  // ~10 s: a phase that never completes traps
+// -DPCC_KCHECK: every slot offset, bulk-copy size / alignment and zero range is asserted (a
+// violation traps); the checked build runs the parity suites (compute-sanitizer is not available)
+#ifdef PCC_KCHECK
+#define PCC_KASSERT(c) \
+    do {               \
+        if (!(c)) __trap(); \
+    } while (0)
+#else
+#define PCC_KASSERT(c) \
+    do {               \
+    } while (0)
+#endif
 
 __device__ __forceinline__ uint32_t sm_addr(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -595,11 +607,13 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
         if (clock64() - t0 > kWaitTrapCycles) __trap();
 }
 __device__ __forceinline__ void bulk_g2s(uint32_t sdst, const void *src, uint32_t bytes, uint32_t bar) {
+    PCC_KASSERT(bytes > 0 && bytes % 16 == 0 && sdst % 16 == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0);
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(sdst),
                  "l"(src), "r"(bytes), "r"(bar)
                  : "memory");
 }
 __device__ __forceinline__ void bulk_s2g(void *dst, uint32_t ssrc, uint32_t bytes) {
+    PCC_KASSERT(bytes > 0 && bytes % 16 == 0 && ssrc % 16 == 0 && (reinterpret_cast<uintptr_t>(dst) & 15) == 0);
     asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(ssrc), "r"(bytes)
                  : "memory");
 }
@@ -664,6 +678,7 @@ __device__ __forceinline__ uint32_t crc_tile_rot(const char *sl, const char *t2,
 }
 
 __device__ __forceinline__ void zero_smem(char *sl, uint32_t a, uint32_t b, uint32_t lane) {  // [a, b), 16-B aligned
+    PCC_KASSERT(a % 16 == 0 && b % 16 == 0 && (a >= b || b <= kTile));
     for (uint32_t o = a + 16 * lane; o < b; o += 512) *reinterpret_cast<uint4 *>(sl + o) = make_uint4(0, 0, 0, 0);
 }
 
@@ -685,9 +700,11 @@ struct ItemGeo {
     __device__ __forceinline__ ItemGeo(const SnapParams &P, uint32_t jl, uint32_t t) {
         j = P.first + jl;
         tile0 = (uint64_t)t * kTile;
+        PCC_KASSERT(t < P.tpc && jl < P.count && tile0 < P.chunk_bytes);
         const uint64_t rem = P.chunk_bytes - tile0;
         len = rem < kTile ? (uint32_t)rem : kTile;
         lead = kTile - len;
+        PCC_KASSERT(len % 16 == 0 && len > 0);
     }
 };
 
@@ -734,6 +751,7 @@ __device__ __forceinline__ Piece piece_of(const SegRow &r, const ItemGeo &g) {
     p.n = p.ok ? (uint32_t)(hi - lo) : 0;
     p.s_off = g.lead + (uint32_t)(lo - g.tile0);
     p.addr = r.ptr + (lo - r.dst_off);
+    PCC_KASSERT(!p.ok || (p.s_off % 16 == 0 && p.s_off >= g.lead && ((p.s_off + p.n + 15) & ~15u) <= kTile));
     return p;
 }
 // slot offset where row i's piece starts (tile end when there is no such row)
