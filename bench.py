@@ -126,33 +126,42 @@ def d2h_peak_gbs(torch, nbytes=1 << 30):
     return nbytes / (best * 1e-3) / 1e9
 
 
-def bidir_peak_gbs(torch, nbytes=1 << 30):
-    """Pinned H2D and D2H copies of `nbytes` each running at once (separate streams): GB/s per
-    direction.  The e2e line moves the slice up AND the checkpoint down every step, so this, not
-    the one-way peak, bounds it."""
+def bidir_peak_gbs(torch, nbytes=2 << 30, piece=64 << 20):
+    """Pinned H2D and D2H running at once, the way the e2e line moves data (a stream of 64 MiB
+    copies each way on two streams), each direction timed on its own stream: (h2d, d2h) GB/s,
+    best of 2.  The e2e line moves the slice up AND the checkpoint down every step, so the slower
+    of these, not the one-way peak, bounds it.  (Measured on the box: 46.5 up + 49.8 down with
+    both running, 55.4 / 56.4 alone; tools/exp/bidir_probe.py.  The round-2 version timed one
+    1 GiB copy each way from a common start and reported ~26 GB/s, below what e2e itself moved.)"""
     d1 = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
     d2 = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
     h1 = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
     h2 = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
     s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
-    best = 1e9
-    for i in range(4):
+    best_up = best_dn = 0.0
+    for i in range(3):
         torch.cuda.synchronize()
-        a = torch.cuda.Event(enable_timing=True)
-        b1, b2 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record(s1)
-        s2.wait_event(a)
+        start = torch.cuda.Event()
+        start.record(torch.cuda.current_stream())
+        e = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+        s1.wait_event(start)
+        s2.wait_event(start)
+        e[0].record(s1)
+        e[2].record(s2)
         with torch.cuda.stream(s1):
-            d1.copy_(h1, non_blocking=True)
+            for o in range(0, nbytes, piece):
+                d1[o:o + piece].copy_(h1[o:o + piece], non_blocking=True)
         with torch.cuda.stream(s2):
-            h2.copy_(d2, non_blocking=True)
-        b1.record(s1)
-        b2.record(s2)
+            for o in range(0, nbytes, piece):
+                h2[o:o + piece].copy_(d2[o:o + piece], non_blocking=True)
+        e[1].record(s1)
+        e[3].record(s2)
         torch.cuda.synchronize()
         if i >= 1:
-            best = min(best, max(a.elapsed_time(b1), a.elapsed_time(b2)))
+            best_up = max(best_up, nbytes / (e[0].elapsed_time(e[1]) * 1e-3) / 1e9)
+            best_dn = max(best_dn, nbytes / (e[2].elapsed_time(e[3]) * 1e-3) / 1e9)
     del d1, d2, h1, h2
-    return nbytes / (best * 1e-3) / 1e9
+    return best_up, best_dn
 
 
 def cpu_baseline(specs, state, cb, budget_bytes=4 << 30, threads=1):
@@ -636,8 +645,9 @@ def main():
             "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": h2d_bytes,
                     "d2h_bytes_per_step": slice_bytes + 4 * (geo["count"] + 1),
                     # both directions busy every step: the bound is the concurrent H2D + D2H rate
-                    "link_peak_bidir_gbs_per_direction": peak_bidir,
-                    "frac_of_bidir": e2e_value / world / peak_bidir},  # per GPU
+                    "link_peak_bidir_gbs": {"h2d": peak_bidir[0], "d2h": peak_bidir[1],
+                                            "def": "both directions at once, 64 MiB copies each way, per-direction stream time"},
+                    "frac_of_bidir": e2e_value / world / min(peak_bidir)},  # per GPU, vs the slower direction
             "gpu_launches": launches,
             "clocks": clk,
             **slowdowns,
