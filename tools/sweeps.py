@@ -37,7 +37,8 @@ def snapshot_rate(pcc, torch, ts, path, cb, flags, n_ckpt=4, n_inflight=2, write
     if path and os.path.exists(path):
         os.unlink(path)
     state = sum(t.numel() * t.element_size() for t in ts)
-    return {"gbs": state * n_ckpt / dt / 1e9, "ms_per_ckpt": dt / n_ckpt * 1e3, "k1_ms": inf["pack_ms"]}
+    return {"gbs": state * n_ckpt / dt / 1e9, "ms_per_ckpt": dt / n_ckpt * 1e3, "k1_ms": inf["k1_busy_ms"],
+            "gate_ms": inf["pack_ms"]}
 
 
 def main():
@@ -56,9 +57,13 @@ def main():
     if not only or "fig12" in only:
         for every in ([1, 2, 5, 10] if not a.quick else [1, 10]):
             for n in [1, 2, 4]:
-                r = vgg16_slowdown(pcc, iters=40 if every < 10 else 60, every=every, runs=1, n_inflight=n)
-                emit({"sweep": "fig12", "every": every, "N": n, "slowdown_pct": r["slowdown_pct"],
-                      "iter_ms_no_ckpt": r["iter_ms_no_ckpt"], "iter_ms_ckpt": r["iter_ms_ckpt"], "p99_ms": r["p99_ms"]})
+                for pace in ("auto", 0.0):  # the tuner's eager pace, and unpaced
+                    r = vgg16_slowdown(pcc, iters=200 if not a.quick else 60, every=every, runs=1, n_inflight=n,
+                                       d2h_gbs=pace)
+                    emit({"sweep": "fig12", "every": every, "N": n, "pace": pace, "d2h_gbs": r.get("d2h_gbs"),
+                          "slowdown_pct": r["slowdown_pct"], "iter_ms_no_ckpt": r["iter_ms_no_ckpt"],
+                          "iter_ms_ckpt": r["iter_ms_ckpt"], "p99_ms": r["p99_ms"],
+                          "pace_delivered_frac": r.get("pace_delivered_frac")})
 
     specs = config_tensors("c2")
     ts = make_state(specs, "cuda", seed=0, it=0)
