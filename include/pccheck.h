@@ -199,6 +199,9 @@ PCC_API int pcc_checkpoint(pcc_ctx *ctx, uint64_t iter, void *train_stream, pcc_
  * profiles/r02_gate_probe_*.txt).  No-op before any checkpoint. */
 PCC_API int pcc_guard(pcc_ctx *ctx, void *train_stream);
 
+/* Handles stay valid until pcc_close: pcc_poll / pcc_wait answer for every handle ever returned
+ * (the outcome of an old terminal checkpoint is kept in 16 bytes); pcc_info keeps the full record
+ * of the newest 64 terminal checkpoints and returns -PCC_EINVAL ("record pruned") for older ones. */
 PCC_API int pcc_poll(pcc_ctx *ctx, pcc_handle h, int *state);
 
 /* Blocks until the checkpoint reached LOCAL_COMMIT (or OBSOLETE / FAILED); timeout_us < 0 =

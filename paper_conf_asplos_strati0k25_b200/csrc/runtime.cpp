@@ -29,6 +29,7 @@
 #include <cstring>
 #include <deque>
 #include <map>
+#include <unordered_map>
 #include <memory>
 #include <mutex>
 #include <set>
@@ -230,6 +231,13 @@ struct pcc_ctx {
     std::mutex ck_mu;
     std::condition_variable ck_cv;
     std::map<uint64_t, std::shared_ptr<Ckpt>> ckpts;  // handle (= counter) -> record
+    // terminal records pruned by gc_ckpts: handle -> outcome, so pcc_poll / pcc_wait still answer
+    // for every handle until close (16 B per checkpoint; pcc_info needs the full record)
+    struct Outcome {
+        int state, err;
+        uint64_t iter;
+    };
+    std::unordered_map<uint64_t, Outcome> pruned;
 
     // threads: packer (K1 windows, in checkpoint order), orchestrator (D2H), persist pool
     BlockingQueue<std::shared_ptr<Ckpt>> packs;
@@ -632,6 +640,7 @@ void gc_ckpts(pcc_ctx *c) {
                         s == PCC_ST_FAILED;
             if (term && it->second->remaining.load() == 0) {
                 dead.push_back(it->second);
+                c->pruned[it->first] = {s, it->second->err.load(), it->second->t.iter};
                 it = c->ckpts.erase(it);
                 --excess;
             } else {
@@ -1147,10 +1156,29 @@ static bool terminal(int s) {
     return s == PCC_ST_LOCAL_COMMIT || s == PCC_ST_GLOBAL_COMMIT || s == PCC_ST_OBSOLETE || s == PCC_ST_FAILED;
 }
 
+// outcome of a pruned terminal handle (false: never issued)
+static bool find_pruned(pcc_ctx *c, pcc_handle h, pcc_ctx::Outcome *o) {
+    std::lock_guard<std::mutex> lk(c->ck_mu);
+    auto it = c->pruned.find(h);
+    if (it == c->pruned.end()) return false;
+    *o = it->second;
+    return true;
+}
+
 int pcc_poll(pcc_ctx *c, pcc_handle h, int *state) {
     if (!c || !state) return set_error(PCC_EINVAL, "args");
     auto ck = find_ck(c, h);
-    if (!ck) return set_error(PCC_EINVAL, "unknown handle");
+    if (!ck) {
+        pcc_ctx::Outcome o;
+        if (!find_pruned(c, h, &o)) return set_error(PCC_EINVAL, "unknown handle");
+        int s = o.state;
+        if (s == PCC_ST_LOCAL_COMMIT && c->cfg.world > 1) {
+            uint64_t g = c->engine->global_iter();
+            if (g != UINT64_MAX && g >= o.iter) s = PCC_ST_GLOBAL_COMMIT;
+        }
+        *state = s;
+        return PCC_OK;
+    }
     int s = ck->state.load();
     if (s == PCC_ST_PACKING && ck->packed_recorded.load() && cudaEventQuery(ck->ev_packed) == cudaSuccess)
         s = PCC_ST_PACKED;
@@ -1165,7 +1193,12 @@ int pcc_poll(pcc_ctx *c, pcc_handle h, int *state) {
 int pcc_wait(pcc_ctx *c, pcc_handle h, int64_t timeout_us) {
     if (!c) return set_error(PCC_EINVAL, "ctx");
     auto ck = find_ck(c, h);
-    if (!ck) return set_error(PCC_EINVAL, "unknown handle");
+    if (!ck) {  // a pruned handle is terminal: its outcome
+        pcc_ctx::Outcome o;
+        if (!find_pruned(c, h, &o)) return set_error(PCC_EINVAL, "unknown handle");
+        if (o.state == PCC_ST_FAILED) return o.err ? o.err : -PCC_EIO;
+        return PCC_OK;
+    }
     std::unique_lock<std::mutex> lk(c->ck_mu);
     auto pred = [&] { return terminal(ck->state.load()); };
     if (timeout_us < 0)
@@ -1239,7 +1272,11 @@ int pcc_commit(pcc_ctx *c, uint64_t *committed_iter) {
 int pcc_info(pcc_ctx *c, pcc_handle h, pcc_ckpt_info *info, uint32_t *crc, uint32_t crc_cap) {
     if (!c || !info) return set_error(PCC_EINVAL, "args");
     auto ck = find_ck(c, h);
-    if (!ck) return set_error(PCC_EINVAL, "unknown handle");
+    if (!ck) {
+        pcc_ctx::Outcome o;
+        return set_error(PCC_EINVAL, find_pruned(c, h, &o) ? "record pruned (pcc_info keeps the newest 64 terminal checkpoints)"
+                                                          : "unknown handle");
+    }
     std::memset(info, 0, sizeof(*info));
     info->iter = ck->t.iter;
     info->counter = ck->t.counter;
@@ -1314,6 +1351,7 @@ int pcc_close(pcc_ctx *c) {
         std::lock_guard<std::mutex> lk(c->ck_mu);
         for (auto &kv : c->ckpts) destroy_ckpt_events(c, kv.second.get());
         c->ckpts.clear();
+        c->pruned.clear();
     }
     free_registration(c);
     for (auto e : c->evpool) cudaEventDestroy(e);

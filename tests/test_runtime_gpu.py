@@ -366,3 +366,26 @@ print(json.dumps(out))
     rc, it, bad, outs = oracle.restore([shm], 3, [s.nbytes for s in config_tensors("c1")],
                                        [s.code for s in config_tensors("c1")], 256, 4 << 20)
     assert rc == 0 and it == 40
+
+
+def test_handles_valid_until_close(pcc, shm):
+    """handles are valid until close.  80 checkpoints one by one: pcc_wait / pcc_poll
+    still answer for the first (its record pruned down to its outcome), pcc_info keeps the newest
+    64 and reports the older ones as pruned; an unknown handle is still an error."""
+    specs = config_tensors("c1")[:12]
+    ts = make_state(specs, "cuda", seed=5, it=0)
+    with pcc.PCCheck(shm, chunk_bytes=1 << 20, max_inflight=2, flags=pcc.MAPFILE) as ck:
+        ck.register(ts)
+        hs = []
+        for i in range(80):
+            hs.append(ck.checkpoint(i + 1))
+            ck.guard()
+            ck.wait(hs[-1])
+        for h in hs:
+            ck.wait(h)
+            assert pcc.STATE_NAMES[ck.poll(h)] == "LOCAL_COMMIT"
+        assert ck.info(hs[-1])["iter"] == 80
+        with pytest.raises(pcc.PCCError):
+            ck.info(hs[0])
+        with pytest.raises(pcc.PCCError):
+            ck.wait(max(hs) + 1000)

@@ -55,11 +55,13 @@ def main():
     only = set(a.only.split(",")) if a.only else None
 
     if not only or "fig12" in only:
+        from bench import d2h_peak_gbs
+        link = d2h_peak_gbs(torch)  # the tuner's link rate, measured here as bench.py does
         for every in ([1, 2, 5, 10] if not a.quick else [1, 10]):
             for n in [1, 2, 4]:
                 for pace in ("auto", 0.0):  # the tuner's eager pace, and unpaced
                     r = vgg16_slowdown(pcc, iters=200 if not a.quick else 60, every=every, runs=1, n_inflight=n,
-                                       d2h_gbs=pace)
+                                       d2h_gbs=pace, link_gbs=link)
                     emit({"sweep": "fig12", "every": every, "N": n, "pace": pace, "d2h_gbs": r.get("d2h_gbs"),
                           "slowdown_pct": r["slowdown_pct"], "iter_ms_no_ckpt": r["iter_ms_no_ckpt"],
                           "iter_ms_ckpt": r["iter_ms_ckpt"], "p99_ms": r["p99_ms"],
