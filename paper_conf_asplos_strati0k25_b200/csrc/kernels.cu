@@ -689,9 +689,6 @@ struct DescBatch {
     uint2 tr;    // x = first row index, y = rows overlapping the tile
     SegRow r0;   // first row (valid when tr.y > 0)
 };
-__device__ __forceinline__ uint2 desc_tr(const SnapParams &P, uint32_t item, uint32_t n_items) {
-    return item_rows(P, item, n_items);
-}
 
 // Geometry of an item (chunk-local index jl, tile t): chunk, tile start, bytes, lead of its slot
 struct ItemGeo {
@@ -963,16 +960,16 @@ __global__ void __launch_bounds__(kTmaThreads, 1) k_snap_tma(const SnapParams P)
     DescBatch cur{}, nxt{};
     uint2 tr_nn = make_uint2(0, 0);
     if (need_desc) {
-        cur.tr = desc_tr(P, batch_item(lane), n_items);
+        cur.tr = item_rows(P, batch_item(lane), n_items);
         if (cur.tr.y) cur.r0 = ld_row(P.rows + cur.tr.x);
-        nxt.tr = desc_tr(P, batch_item(32 + lane), n_items);
+        nxt.tr = item_rows(P, batch_item(32 + lane), n_items);
     }
     RoleIter it(P, r, nr);
     uint32_t m = 0;  // this warp's item count
     for (uint32_t b = 0; it.item < n_items; ++b) {
         if (need_desc) {  // first rows of the next batch, row ranges of the one after
             if (nxt.tr.y) nxt.r0 = ld_row(P.rows + nxt.tr.x);
-            tr_nn = desc_tr(P, batch_item(32 * (b + 2) + lane), n_items);
+            tr_nn = item_rows(P, batch_item(32 * (b + 2) + lane), n_items);
         }
         for (uint32_t ii = 0; ii < 32 && it.item < n_items; ++ii, ++m, it.next()) {
             const uint32_t k = it.k, s = k % kStages, use = k / kStages;
