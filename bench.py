@@ -561,8 +561,16 @@ def main():
         rit, rbad = ck.restore()
         torch.cuda.synchronize()
         rdt = time.perf_counter() - t0r
+        rs = ck.restore_stats()
         restore = {"iter": rit, "ms": rdt * 1e3, "gbs": state_bytes / rdt / 1e9, "bad_chunks": len(rbad),
-                   "path": "file mapping -> H2D into the HBM ring -> K2 verify+scatter"}
+                   "path": "file mapping -> H2D into the HBM ring -> K2 verify+scatter",
+                   # SURVEY §8(d) breakdown (pcc_restore_stats; storage read is the copy engine's
+                   # read of the mapped file, inside h2d, in MAPFILE mode)
+                   "breakdown_ms": {k: rs[k] for k in ("read_ms", "h2d_ms", "k2_ms", "finalize_ms", "fanout_ms",
+                                                       "total_ms")},
+                   "h2d_gbs": rs["bytes"] / (rs["h2d_ms"] * 1e-3) / 1e9 if rs["h2d_ms"] else None,
+                   # K2 reads the staged slice and writes the state bytes back: bytes + state bytes
+                   "k2_gbs": (rs["bytes"] + state_bytes) / (rs["k2_ms"] * 1e-3) / 1e9 if rs["k2_ms"] else None}
     barrier()  # W > 1: every GPU probes its link at the same time (the peak at the same concurrency)
     peak_link = d2h_peak_gbs(torch)
     peak_bidir = bidir_peak_gbs(torch)
@@ -605,6 +613,8 @@ def main():
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
             peaks = json.load(f)
         k1_bytes = rank_state_bytes + slice_bytes  # read the slice's state bytes + write the packed slice (R3: pads count)
+        if restore and restore.get("k2_gbs"):
+            restore["k2_hbm_frac"] = restore["k2_gbs"] / peaks["hbm_gbs"]
         k1_achieved = k1_bytes / (k1_ms * 1e-3) / 1e9
         link_achieved = slice_bytes / (ms_total * 1e-3 / args.steps) / 1e9
         line = {

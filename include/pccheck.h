@@ -231,6 +231,22 @@ PCC_API int pcc_latest(const char *path, uint64_t *global_iter, uint64_t *local_
 PCC_API int pcc_restore(pcc_ctx *ctx, uint64_t want_iter, uint32_t flags, uint64_t *restored_iter,
                 uint32_t *bad_chunks, uint32_t bad_cap, uint32_t *n_bad);
 
+/* Where the last pcc_restore's time went (storage read, H2D, K2, allgather), this
+ * rank.  Times are summed over every candidate checkpoint the restore tried (fallback). */
+typedef struct {
+    uint64_t bytes;            /* slice bytes read + verified from this rank's file             */
+    uint32_t attempts;         /* candidate checkpoints verified (1 + fallbacks)                 */
+    float total_ms;            /* pcc_restore call -> return (host clock)                        */
+    float read_ms;             /* storage read: pread into pinned staging (host clock); 0 with
+                                  PCC_MAPFILE, where the copy engine reads the mapped file pages */
+    float h2d_ms;              /* first H2D start -> last H2D end (CUDA events, copy stream)     */
+    float k2_ms;               /* the K2 launches over this rank's slice, summed (CUDA events)   */
+    float finalize_ms;         /* chunk CRCs + digest compare (CUDA events)                       */
+    float fanout_ms;           /* world > 1: allgather of the other ranks' chunks + their K2
+                                  (host clock); 0 at world 1                                      */
+} pcc_restore_info;
+PCC_API int pcc_restore_stats(pcc_ctx *ctx, pcc_restore_info *out);
+
 /* Diagnostics of one checkpoint (timings, digest) and its chunk CRC table (crc_cap entries). */
 PCC_API int pcc_info(pcc_ctx *ctx, pcc_handle h, pcc_ckpt_info *info, uint32_t *crc, uint32_t crc_cap);
 

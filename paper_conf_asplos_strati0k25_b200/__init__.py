@@ -49,6 +49,11 @@ class Tensor(C.Structure):
     _fields_ = [("dev_ptr", C.c_void_p), ("nbytes", C.c_uint64), ("dtype", C.c_uint32), ("name", C.c_char_p)]
 
 
+class RestoreInfo(C.Structure):  # pcc_restore_info
+    _fields_ = [("bytes", C.c_uint64), ("attempts", C.c_uint32), ("total_ms", C.c_float), ("read_ms", C.c_float),
+                ("h2d_ms", C.c_float), ("k2_ms", C.c_float), ("finalize_ms", C.c_float), ("fanout_ms", C.c_float)]
+
+
 class Info(C.Structure):
     _fields_ = [("iter", C.c_uint64), ("counter", C.c_uint64), ("slot", C.c_uint32), ("state", C.c_uint32),
                 ("digest", C.c_uint32), ("n_chunks", C.c_uint32), ("t_call_us", C.c_double),
@@ -82,6 +87,7 @@ _SIGS = {
     "pcc_close": (C.c_int, [_P]),
     "pcc_nccl_unique_id": (C.c_int, [_P]),
     "pcc_struct_size": (C.c_uint64, [C.c_int]),
+    "pcc_restore_stats": (C.c_int, [_P, _P]),
     "pcc_strerror": (C.c_char_p, [C.c_int]),
     "pcc_last_error": (C.c_char_p, []),
     "pcc_last_errno": (C.c_int, []),
@@ -258,6 +264,13 @@ class PCCheck:
             err.bad_chunks = bad_list
             raise err
         return it.value, bad_list
+
+    def restore_stats(self):
+        """Where the last restore's time went (pcc_restore_stats): storage read, H2D, K2,
+        finalize, fan-out (W > 1), total — ms, summed over the candidates tried."""
+        r = RestoreInfo()
+        _check(_lib.pcc_restore_stats(self._ctx, C.byref(r)), "pcc_restore_stats")
+        return {f: getattr(r, f) for f, _ in RestoreInfo._fields_}
 
     def info(self, h, with_crc=False):
         inf = Info()

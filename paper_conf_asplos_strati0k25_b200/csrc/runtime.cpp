@@ -238,6 +238,7 @@ struct pcc_ctx {
         uint64_t iter;
     };
     std::unordered_map<uint64_t, Outcome> pruned;
+    pcc_restore_info rstats{};  // the last pcc_restore's breakdown
 
     // threads: packer (K1 windows, in checkpoint order), orchestrator (D2H), persist pool
     BlockingQueue<std::shared_ptr<Ckpt>> packs;
@@ -854,7 +855,11 @@ const char *pcc_strerror(int err) {
     }
 }
 uint64_t pcc_struct_size(int which) {
-    return which == 0 ? sizeof(pcc_config) : which == 1 ? sizeof(pcc_tensor) : which == 2 ? sizeof(pcc_ckpt_info) : 0;
+    return which == 0   ? sizeof(pcc_config)
+           : which == 1 ? sizeof(pcc_tensor)
+           : which == 2 ? sizeof(pcc_ckpt_info)
+           : which == 3 ? sizeof(pcc_restore_info)
+                        : 0;
 }
 const char *pcc_last_error(void) { return err_state().msg.c_str(); }
 int pcc_last_errno(void) { return err_state().err_no; }
@@ -1438,6 +1443,15 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     const bool whole = R >= n;
     const uint64_t batch = whole ? std::max<uint64_t>(1, (n + 3) / 4) : R;
     cudaEvent_t ev_copy = get_event(c), ev_k2 = get_event(c);
+    // timing (pcc_restore_stats): H2D span on the copy stream, each K2 launch and the finalize
+    cudaEvent_t t_h2d[2], t_fin[2];
+    for (auto *e2 : {t_h2d, t_fin}) {
+        cudaEventCreate(&e2[0]);
+        cudaEventCreate(&e2[1]);
+    }
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> t_k2;
+    double read_ms = 0;
+    cudaEventRecord(t_h2d[0], c->copy_stream);
     const uint64_t data0 = c->slot_data_off(slot);
     for (uint64_t j0 = 0; j0 < n && rc == PCC_OK; j0 += batch) {
         const uint64_t k = std::min<uint64_t>(batch, n - j0);
@@ -1450,7 +1464,9 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
             } else {  // pread into a pinned staging slot, then H2D (the slot is reused after the copy)
                 char *st = c->staging + (i % c->staging_slots) * cb;
                 if (i >= c->staging_slots) cudaStreamSynchronize(c->copy_stream);
+                const auto tr0 = std::chrono::steady_clock::now();
                 rc = pread_full(c->fd, st, cb, data0 + j * cb);
+                read_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tr0).count();
                 if (rc == PCC_OK) cudaMemcpyAsync(dst, st, cb, cudaMemcpyHostToDevice, c->copy_stream);
             }
         }
@@ -1460,11 +1476,18 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
         P.first = (uint32_t)j0;
         P.count = (uint32_t)k;
         P.ring_head = whole ? 0 : (R - j0 % R) % R;
+        std::pair<cudaEvent_t, cudaEvent_t> tk;
+        cudaEventCreate(&tk.first);
+        cudaEventCreate(&tk.second);
+        t_k2.push_back(tk);
+        cudaEventRecord(tk.first, c->pack_stream);
         if ((e = launch_unpack(P, snapshot_grid(c->device, (uint32_t)(k * P.tpc), 0, false), c->pack_stream)))
             rc = cuda_error(e, "K2");
+        cudaEventRecord(tk.second, c->pack_stream);
         c->launches += 1;
         cudaEventRecord(ev_k2, c->pack_stream);
     }
+    cudaEventRecord(t_h2d[1], c->copy_stream);
     PCC_TRACE("restore: copies + K2 issued t=%.0f us", c->now_us());
     FinalizeParams F{};
     F.tile_crc = tile;
@@ -1478,7 +1501,9 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     F.expect = expect;
     F.bad = bad;
     F.scratch = scr;
+    cudaEventRecord(t_fin[0], c->pack_stream);
     if (rc == PCC_OK && (e = launch_finalize(F, c->pack_stream))) rc = cuda_error(e, "finalize");
+    cudaEventRecord(t_fin[1], c->pack_stream);
     c->launches += kFinalizeLaunches;
     std::vector<uint32_t> flags(n);
     uint32_t sc[4] = {0, 0, 0, 0};
@@ -1489,6 +1514,24 @@ int verify_scatter(pcc_ctx *c, uint32_t slot, std::vector<uint32_t> *bad_out) {
     }
     cudaStreamSynchronize(c->copy_stream);
     PCC_TRACE("restore: verified t=%.0f us", c->now_us());
+    {
+        pcc_restore_info &st = c->rstats;
+        float ms = 0;
+        st.attempts += 1;
+        st.bytes += n * cb;
+        st.read_ms += (float)read_ms;
+        if (cudaEventElapsedTime(&ms, t_h2d[0], t_h2d[1]) == cudaSuccess) st.h2d_ms += ms;
+        if (cudaEventElapsedTime(&ms, t_fin[0], t_fin[1]) == cudaSuccess) st.finalize_ms += ms;
+        for (auto &tk : t_k2) {
+            if (cudaEventElapsedTime(&ms, tk.first, tk.second) == cudaSuccess) st.k2_ms += ms;
+            cudaEventDestroy(tk.first);
+            cudaEventDestroy(tk.second);
+        }
+        for (auto *e2 : {t_h2d, t_fin}) {
+            cudaEventDestroy(e2[0]);
+            cudaEventDestroy(e2[1]);
+        }
+    }
     put_event(c, ev_copy);
     put_event(c, ev_k2);
     if (own_ring) cudaFree(ring);
@@ -1683,6 +1726,8 @@ extern "C" int pcc_restore(pcc_ctx *c, uint64_t want_iter, uint32_t flags, uint6
     if (c->fd < 0) return set_error(PCC_ENOENT, "no file (NULLSINK)");
     pcc_drain(c, -1);
     cudaSetDevice(c->device);
+    const auto t_start = std::chrono::steady_clock::now();
+    c->rstats = pcc_restore_info{};
     PCC_TRACE("restore: start t=%.0f us", c->now_us());
     SlotScan S;
     int rc = scan_rank_file(c->fd, c->sgeom, c->n_slots, &S);
@@ -1694,7 +1739,13 @@ extern "C" int pcc_restore(pcc_ctx *c, uint64_t want_iter, uint32_t flags, uint6
     } else {
         ops.reduce = [c](int64_t *v, bool is_max) { return reduce_i64(c, v, 1, is_max ? NcclComm::kMax : NcclComm::kMin); };
         if (!(c->cfg.flags & (PCC_NOCOMM | PCC_SHARDED)))
-            ops.fanout = [c](uint64_t, uint32_t slot) { return dp_fanout(c, slot); };
+            ops.fanout = [c](uint64_t, uint32_t slot) {
+                const auto t0 = std::chrono::steady_clock::now();
+                int r = dp_fanout(c, slot);
+                c->rstats.fanout_ms +=
+                    (float)std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+                return r;
+            };
     }
     ops.verify = [c](uint64_t, uint32_t slot, std::vector<uint32_t> *bad) { return verify_scatter(c, slot, bad); };
     uint64_t it = 0;
@@ -1703,5 +1754,13 @@ extern "C" int pcc_restore(pcc_ctx *c, uint64_t want_iter, uint32_t flags, uint6
     if (n_bad) *n_bad = (uint32_t)bad.size();
     for (size_t i = 0; i < bad.size() && i < bad_cap && bad_chunks; ++i) bad_chunks[i] = bad[i];
     if (rc == PCC_OK && restored_iter) *restored_iter = it;
+    c->rstats.total_ms =
+        (float)std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
     return rc;
+}
+
+extern "C" int pcc_restore_stats(pcc_ctx *c, pcc_restore_info *out) {
+    if (!c || !out) return set_error(PCC_EINVAL, "args");
+    *out = c->rstats;
+    return PCC_OK;
 }

@@ -38,6 +38,7 @@ def test_struct_mirrors_match_the_build():
     assert pcc._lib.pcc_struct_size(0) == ctypes.sizeof(pcc.Config)
     assert pcc._lib.pcc_struct_size(1) == ctypes.sizeof(pcc.Tensor)
     assert pcc._lib.pcc_struct_size(2) == ctypes.sizeof(pcc.Info)
+    assert pcc._lib.pcc_struct_size(3) == ctypes.sizeof(pcc.RestoreInfo)
     assert pcc._lib.pcc_struct_size(7) == 0
 
 

@@ -162,6 +162,13 @@ def test_restore_roundtrip_and_faults(pcc, shm, mode):
         it, bad = ck.restore()
         assert it == 20 and bad == []
         assert all(np.array_equal(host_bytes(t), s) for t, s in zip(ts, s20))
+        # pcc_restore_stats: the breakdown of that restore
+        rs = ck.restore_stats()
+        c = ck.geometry()["count"]
+        assert rs["attempts"] == 1 and rs["bytes"] == c * cb
+        assert rs["h2d_ms"] > 0 and rs["k2_ms"] > 0 and rs["finalize_ms"] > 0 and rs["fanout_ms"] == 0
+        assert rs["total_ms"] >= rs["k2_ms"] and rs["total_ms"] >= rs["read_ms"]
+        assert (rs["read_ms"] > 0) == (mode != "mapfile")  # MAPFILE: the copy engine reads the mapping
         # corrupt chunk 3 of iter 20's slot: one bit
         inf = ck.info(h20)
         c = ck.geometry()["count"]
@@ -177,6 +184,8 @@ def test_restore_roundtrip_and_faults(pcc, shm, mode):
         it, bad = ck.restore(fallback=True)
         assert it == 10
         assert all(np.array_equal(host_bytes(t), s) for t, s in zip(ts, s10))
+        rs = ck.restore_stats()
+        assert rs["attempts"] == 2 and rs["bytes"] == 2 * c * cb  # iter 20 rejected, then iter 10
 
 
 def test_nullsink_and_launch_count(pcc):
