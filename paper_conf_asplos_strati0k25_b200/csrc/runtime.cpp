@@ -749,12 +749,14 @@ void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
         while (done < c->n && e == cudaSuccess) {
             uint64_t k;
             {
-                // launch windows of at least a quarter ring (or the rest of the slice): when the
+                // launch windows of at least half the ring (or the rest of the slice): when the
                 // link is the bottleneck the ring frees a chunk or two at a time, and a K1 launch
                 // per freed chunk pays the table load and launch latency each time (C3 with
                 // N = 4 over a 2-slice ring: 114 launches per checkpoint, 11.7 ms of K1 instead
-                // of 5.7).  The chunks already packed keep the copy engine busy meanwhile.
-                const uint64_t want = std::min<uint64_t>(c->n - done, std::max<uint64_t>(1, c->ring_slots / 4));
+                // of 5.7).  The chunks already packed keep the copy engine busy meanwhile.  Half
+                // (round 2; a quarter before): a 2-slice ring packs each back-to-back checkpoint
+                // in one launch (1.9 before), a 1-slice ring in at most two.
+                const uint64_t want = std::min<uint64_t>(c->n - done, std::max<uint64_t>(1, c->ring_slots / 2));
                 std::unique_lock<std::mutex> lk(c->ring_mu);
                 c->ring_cv.wait(lk, [&] { return c->ring_tail + c->ring_slots >= ck->ring_start + done + want; });
                 k = std::min<uint64_t>(c->n - done, c->ring_tail + c->ring_slots - (ck->ring_start + done));
