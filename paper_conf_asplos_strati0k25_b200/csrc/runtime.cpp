@@ -454,10 +454,13 @@ void orchestrate_loop(pcc_ctx *c) {
     // 0.5 MiB quanta a per-copy count drained every 1 MiB and the host round trips capped the
     // paced transfer at ~9.5 GB/s against a 28.6 GB/s target.  A paced transfer
     // never drains: its own gaps already let other streams' copies through.
-    static const uint64_t d2h_drain = [] {
+    // With small unpaced copies (d2h_quantum <= 2 MiB: the tuner's choice under an eager loop)
+    // the queue drains every 16 MiB: eager OPT-1.3B 8.8% -> 7.6% (profiles/r02e2_eager_piece.jsonl).
+    static const uint64_t d2h_drain_env = [] {
         const char *e = std::getenv("PCC_D2H_DRAIN_MIB");
-        return (e ? std::strtoull(e, nullptr, 10) : 128ull) << 20;  // 0 = never
+        return e ? std::strtoull(e, nullptr, 10) << 20 : ~0ull;  // 0 = never
     }();
+
     uint64_t since_drain = 0;
     std::deque<cudaEvent_t> queued;  // completion events of the pieces on the copy engine
     // waited for by polling cudaEventQuery between yields: cudaEventSynchronize's spin delayed
@@ -481,6 +484,9 @@ void orchestrate_loop(pcc_ctx *c) {
         // issued no faster than `pace` bytes per microsecond once the chunks exist in HBM
         const uint64_t pace = c->cfg.d2h_mbps;  // MB/s == bytes per microsecond
         const uint64_t quantum = c->cfg.d2h_quantum;
+        const uint64_t d2h_drain = d2h_drain_env != ~0ull                      ? d2h_drain_env
+                                   : (quantum && quantum <= (2ull << 20)) ? (16ull << 20)
+                                                                          : (128ull << 20);
         Clock::time_point t_pace{};
         bool pace_started = false;
         uint64_t paced_bytes = 0;

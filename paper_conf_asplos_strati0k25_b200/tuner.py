@@ -84,6 +84,7 @@ D2H_QUANTUM = 1 << 20    # bytes per paced copy (1 MiB: r02 sweeps, eager and gr
 EAGER_MARGIN, EAGER_CAP = 0.9, 0.7   # eager loop: land within 0.9 of the interval, pace <= 0.7 x link
 GRAPH_MARGIN, GRAPH_CAP = 0.85, 0.85  # CUDA-graph loop
 GRAPH_QUANTUM = D2H_QUANTUM
+UNPACED_EAGER_QUANTUM = 1 << 20  # unpaced copies under an eager loop (the runtime then drains every 16 MiB)
 
 
 def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, n_inflight: int = 2,
@@ -100,7 +101,9 @@ def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, n_inflight:
       unpaced 3.9%; 35 / 45 GB/s in 1 MiB copies 1.1 / 1.8%; 4 MiB copies 3.0-3.3%.  A replay pays
       per byte in flight on the link, so a long gentle transfer in small copies is cheap:
       margin 0.85, cap 0.85 of the link.
-    * eager loop (OPT-1.3B, 10 x 44 ms, profiles/r02_eager_pace.jsonl): unpaced 18.9%; 40 GB/s in
+    * eager loop (OPT-1.3B, 10 x 44 ms, profiles/r02_eager_pace.jsonl): unpaced 18.9% (in 64 MiB
+      copies; 1 MiB copies, draining every 16 MiB: 7.6%, which is what an unpaced eager choice
+      gets); 40 GB/s in
       1 MiB copies 6.5%; 50 GB/s 63% — near the link the copy queue never runs dry and the
       training's own small D2H (HF's per-forward flag read) waits behind it (the r01 starvation);
       256 KiB copies: the host cannot keep the cadence (0.57 of the pace delivered).  Margin 0.9,
@@ -115,7 +118,10 @@ def choose_pace(slice_bytes: int, f: int, t: float, link_gbs: float, n_inflight:
     need = slice_bytes / (margin * f * t) / 1e9  # GB/s to land a checkpoint in margin * f * t
     g = min(max(need, 0.5 * link_gbs), cap * link_gbs)
     if slice_bytes / (g * 1e9) > f * t:  # even the capped pace outlasts the interval: unpaced
-        return {"d2h_gbs": 0.0, "d2h_quantum": 0, "need_gbs": need}
+        # ... but an eager loop still gets 1 MiB copies: its extra time per burst iteration
+        # follows the copy size (OPT-1.3B unpaced: 20.8% in 64 MiB copies, 8.8% in 1 MiB;
+        # profiles/r02e2_eager_piece.jsonl).  A CUDA-graph loop keeps whole chunk groups.
+        return {"d2h_gbs": 0.0, "d2h_quantum": 0 if graphs else UNPACED_EAGER_QUANTUM, "need_gbs": need}
     return {"d2h_gbs": g, "d2h_quantum": D2H_QUANTUM, "need_gbs": need}
 
 

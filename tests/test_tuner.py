@@ -27,7 +27,7 @@ def test_choose_pace():
     assert 28.5 < p["d2h_gbs"] <= 0.7 * 57.0 and p["d2h_gbs"] == pytest.approx(min(p["need_gbs"], 0.7 * 57.0))
     # even the capped pace outlasts the interval (every iteration): unpaced
     p = choose_pace(1_107_296_256, 1, 0.0171, 57.0)
-    assert p["d2h_gbs"] == 0.0 and p["d2h_quantum"] == 0
+    assert p["d2h_gbs"] == 0.0 and p["d2h_quantum"] == 1 << 20  # unpaced, but in 1 MiB copies (eager)
     # OPT-1.3B eager (15.8 GB every 10 x 44 ms) needs 39.9 GB/s at margin 0.9: on a 57.1 GB/s link
     # that is under the cap; on a 56.0 GB/s link it is capped at 39.2 GB/s, which still lands in
     # 403 ms < 440 ms
@@ -46,7 +46,8 @@ def test_choose_pace():
     p = choose_pace(15_789_098_512, 10, 0.0517, 56.7, graphs=True)
     assert p["d2h_gbs"] == pytest.approx(15_789_098_512 / (0.85 * 10 * 0.0517) / 1e9) and p["d2h_quantum"] == 1 << 20
     assert 28.35 < p["d2h_gbs"] < 0.85 * 56.7
-    assert choose_pace(15_789_098_512, 4, 0.0517, 56.7, graphs=True)["d2h_gbs"] == 0.0  # would outlast the interval
+    p = choose_pace(15_789_098_512, 4, 0.0517, 56.7, graphs=True)  # would outlast the interval
+    assert p["d2h_gbs"] == 0.0 and p["d2h_quantum"] == 0  # graphs keep whole chunk groups
 
 
 @pytest.mark.gpu
