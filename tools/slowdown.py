@@ -410,6 +410,7 @@ if __name__ == "__main__":
     ap.add_argument("--pack-ctas", type=int, default=0)
     ap.add_argument("--no-upfront", action="store_true", help="graphs: keep the orchestrator-issued (pace-able) D2H")
     ap.add_argument("--quantum-kib", type=int, default=512)
+    ap.add_argument("--unpaced-quantum-kib", type=int, default=0, help="copy size of an unpaced D2H (0 = whole chunk groups)")
     ap.add_argument("--ring-slices", type=float, default=0, help="HBM ring in slices (0 = one slice)")
     a = ap.parse_args()
     import paper_conf_asplos_strati0k25_b200 as pcc
@@ -427,5 +428,5 @@ if __name__ == "__main__":
             ring = int(a.ring_slices * -(-nb // (64 << 20))) * (64 << 20)
         r = hf_slowdown(pcc, a.model, graphs=a.graphs, host_lead=a.host_lead or None, n_inflight=a.inflight,
                         ring_bytes=ring, pack_ctas=a.pack_ctas, upfront=False if a.no_upfront else None,
-                        d2h_quantum=(a.quantum_kib << 10) if pace else 0, **kw)
+                        d2h_quantum=(a.quantum_kib << 10) if pace else (a.unpaced_quantum_kib << 10), **kw)
     print(json.dumps(r))
