@@ -762,7 +762,11 @@ void pack_one(pcc_ctx *c, const std::shared_ptr<Ckpt> &ck) {
                 // of 5.7).  The chunks already packed keep the copy engine busy meanwhile.  Half
                 // (round 2; a quarter before): a 2-slice ring packs each back-to-back checkpoint
                 // in one launch (1.9 before), a 1-slice ring in at most two.
-                const uint64_t want = std::min<uint64_t>(c->n - done, std::max<uint64_t>(1, c->ring_slots / 2));
+#ifndef PCC_RING_WINDOW_DIV  // A/B hook: 4 = the earlier quarter-ring rule
+#define PCC_RING_WINDOW_DIV 2
+#endif
+                const uint64_t want =
+                    std::min<uint64_t>(c->n - done, std::max<uint64_t>(1, c->ring_slots / PCC_RING_WINDOW_DIV));
                 std::unique_lock<std::mutex> lk(c->ring_mu);
                 c->ring_cv.wait(lk, [&] { return c->ring_tail + c->ring_slots >= ck->ring_start + done + want; });
                 k = std::min<uint64_t>(c->n - done, c->ring_tail + c->ring_slots - (ck->ring_start + done));
