@@ -59,6 +59,9 @@ def _rank_main(rank, world, tmpdir, port, q, transport="gloo"):
             it, bad = ck.restore()
             out["restore"] = it
             out["restore_ok"] = all(np.array_equal(host_bytes(t), s) for t, s in zip(ts, saved[30]))
+            rs = ck.restore_stats()  # pcc_restore_stats at W = 2: the fan-out is timed too
+            out["restore_stats_ok"] = (rs["attempts"] == 1 and rs["bytes"] == geo["count"] * CB and rs["fanout_ms"] > 0
+                                       and rs["k2_ms"] > 0 and rs["total_ms"] >= rs["fanout_ms"])
             # rank 1's newest slice is corrupted -> every rank must reject 30 and agree on 20
             dist.barrier()
             if rank == 1:
@@ -130,7 +133,7 @@ def test_dp_world2(shmdir, transport):
     assert res[0]["slice"] == (0, 8, 17) and res[1]["slice"] == (8, 9, 17)
     for r in range(2):
         assert (res[r]["g10"], res[r]["g20"], res[r]["g30"]) == (10, 20, 30)
-        assert res[r]["restore"] == 30 and res[r]["restore_ok"]
+        assert res[r]["restore"] == 30 and res[r]["restore_ok"] and res[r]["restore_stats_ok"]
         assert res[r]["corrupt_rc"] == pcc.ECORRUPT
         assert res[r]["fallback"] == 20 and res[r]["fallback_ok"]
     # the oracle, reading both rank files, agrees (with fallback past the corrupted slice)
